@@ -1,0 +1,355 @@
+#!/usr/bin/env python3
+"""bench.py -- BPBC Smith-Waterman on B200: GCUPS with bit-exact max local scores.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2] [--impl ours|reference]
+
+One "step" = the whole hot path (W2B pack of query and target -> bit-sliced
+wavefront sweep -> max reduction + B2W untranspose) over one
+batch of synthetic pairs already resident in HBM.  Default workload (N=1) is
+BASELINE.json configs[1] = C2: 2^20 DNA pairs, m = n = 128, +2/-1/-1, 9-bit
+slices.  For N > 1 (torchrun, one process per GPU) every rank scores its own
+C2-sized shard (weak scaling, no collective on the data path) and the
+per-step result gather is an NCCL all_gather of the int32 scores.
+
+Prints ONE JSON line on rank 0 (contract in the task statement / DESIGN.md
+"Measurement"): metric, value (GCUPS, all ranks), e2e (same metric through
+the host-buffer C call bpbc_sw_score_batch_host with pinned host inputs,
+H2D + D2H inside the timed region), roofline (the sweep kernel against the
+integer-logic pipe peak), cpu_baseline (the oracle on a bounded sample on
+this host's cores), clocks (nvidia-smi sampled during the timed region),
+gpu_launches, parity (a sample of pairs checked against the oracle).
+
+--impl reference times the CPU oracle (oracle/) on the same config -- the
+reference arm of this tier (no reference implementation exists).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "GCUPS (bit-exact max local score)"
+CONFIGS = {
+    1: dict(P=1024, m=64, n=64, s=8),
+    2: dict(P=1 << 20, m=128, n=128, s=9),
+    3: dict(P=1 << 22, m=256, n=256, s=10),
+    4: dict(P=1 << 20, m=64, n=1024, s=8),
+}
+CONSTS = (2, -1, -1)  # match, mismatch, gap (Table II, reading R14)
+SM_COUNT = 148
+ALU_LANES_PER_SM_CLK = 64  # 4 SMSP x 16 lanes/clk (LOP3 rt = 2 cyc per warp instr)
+
+
+def workload_name(cid, c):
+    return (f"C{cid}: {c['P']} DNA pairs, m={c['m']}, n={c['n']}, "
+            f"match/mismatch/gap = +2/-1/-1, {c['s']}-bit score slices, max score only")
+
+
+def survey_ops_per_word_cell(s):
+    """LOP3 form of the circuit, 11s + 2 per 32-cell word."""
+    return 11 * s + 2
+
+
+def peak_alu_tops(sm_mhz):
+    return SM_COUNT * ALU_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.thread.join(timeout=2)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_baseline(cfg, target_seconds=12.0):
+    """The oracle as it stands, on a bounded sample of the workload, all host cores."""
+    import oracle
+    import synth
+    threads = os.cpu_count() or 1
+    m, n = cfg["m"], cfg["n"]
+    seed = synth.seed_for_config(cfg["id"])
+    cal = max(threads, 256)
+    q, t = synth.gen_pairs(seed, cal, m, n)
+    t0 = time.perf_counter()
+    oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
+    rate = cal / max(time.perf_counter() - t0, 1e-6)
+    sample = int(min(cfg["P"], max(threads, rate * target_seconds)))
+    q, t = synth.gen_pairs(seed, sample, m, n)
+    t0 = time.perf_counter()
+    oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
+    dt = time.perf_counter() - t0
+    return {"value": round(sample * m * n / dt / 1e9, 4), "unit": "GCUPS", "cores": threads,
+            "kind": "oracle",
+            "sample": f"first {sample} of the {cfg['P']} pairs of C{cfg['id']} "
+                      f"(m={m}, n={n}), {dt:.1f} s, scalar int32 DP, {threads} threads"}
+
+
+def run_reference(args, cfg):
+    """--impl reference: the CPU oracle timed on this host (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    import synth
+    threads = os.cpu_count() or 1
+    m, n = cfg["m"], cfg["n"]
+    seed = synth.seed_for_config(cfg["id"])
+    # size one step so the whole run stays within ~1-2 minutes
+    cal = max(threads, 256)
+    q, t = synth.gen_pairs(seed, cal, m, n)
+    t0 = time.perf_counter()
+    oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
+    rate = cal / max(time.perf_counter() - t0, 1e-6)
+    per_step = int(min(cfg["P"], max(threads, rate * 60.0 / max(1, args.steps + args.warmup))))
+    q, t = synth.gen_pairs(seed, per_step, m, n)
+    for _ in range(args.warmup):
+        oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
+    dt = time.perf_counter() - t0
+    v = per_step * m * n * args.steps / dt / 1e9
+    line = {"metric": METRIC, "value": round(v, 4), "unit": "GCUPS", "impl": "reference",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": workload_name(cfg["id"], cfg),
+                       "sample_pairs_per_step": per_step},
+            "cpu_baseline": {"value": round(v, 4), "unit": "GCUPS", "cores": threads,
+                             "kind": "oracle",
+                             "sample": f"{per_step} pairs of C{cfg['id']} per step"},
+            "e2e": {"value": round(v, 4), "unit": "GCUPS", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=2, choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--score-bits", type=int, default=None)
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "ours":
+        print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
+    cfg = dict(CONFIGS[args.config])
+    cfg["id"] = args.config
+    if args.score_bits:
+        cfg["s"] = args.score_bits
+    if args.impl == "reference":
+        run_reference(args, cfg)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    import paper_conf_ipps_nishimurabin17_b200 as bpbc
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    P, m, n, s = cfg["P"], cfg["m"], cfg["n"], cfg["s"]
+    seed = synth.seed_for_config(args.config)
+
+    # inputs: this rank's shard, generated on the host into pinned buffers
+    hq = torch.empty((P, m), dtype=torch.uint8, pin_memory=True)
+    ht = torch.empty((P, n), dtype=torch.uint8, pin_memory=True)
+    synth.gen_pairs(seed, P, m, n, p_offset=rank * P, out_q=hq.numpy(), out_t=ht.numpy())
+    dq = hq.to(dev, non_blocking=True)
+    dt = ht.to(dev, non_blocking=True)
+    out = torch.empty(P, dtype=torch.int32, device=dev)
+    ws = torch.empty(bpbc.workspace_bytes(P, m, n), dtype=torch.uint8, device=dev)
+    gathered = torch.empty(world * P, dtype=torch.int32, device=dev) if world > 1 else None
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    torch.cuda.synchronize()
+
+    def step():
+        bpbc.score_batch(dq, dt, *CONSTS, score_bits=s, out=out, workspace=ws)
+        if gathered is not None:
+            dist.all_gather_into_tensor(gathered, out)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    plan = bpbc.last_plan(local)
+
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    sampler = ClockSampler(local).start()
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    bpbc.profile(True, local)
+    for k in range(args.steps):
+        flush.zero_()  # L2 flush between timed steps (outside the events)
+        starts[k].record()
+        step()
+        ends[k].record()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    phases = bpbc.profile_read(local)
+    bpbc.profile(False, local)
+    t_ms = sum(a.elapsed_time(b) for a, b in zip(starts, ends))
+    if world > 1:
+        tt = torch.tensor([t_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_ms = tt.item()
+    cells = world * P * m * n * args.steps
+    gcups = cells / (t_ms / 1e3) / 1e9
+
+    # ---------------- end to end through the host-buffer C call
+    e2e = None
+    if not args.no_e2e:
+        hout = torch.empty(P, dtype=torch.int32, pin_memory=True)
+        qn, tn, on = hq.numpy(), ht.numpy(), hout.numpy()
+        for _ in range(2):
+            bpbc.score_batch_host(qn, tn, *CONSTS, score_bits=s, device=local, out=on)
+        if world > 1:
+            dist.barrier()
+        ksteps = max(3, min(args.steps, 10))
+        t0 = time.perf_counter()
+        for _ in range(ksteps):
+            bpbc.score_batch_host(qn, tn, *CONSTS, score_bits=s, device=local, out=on)
+        el = time.perf_counter() - t0
+        if world > 1:
+            te = torch.tensor([el], dtype=torch.float64, device=dev)
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+            el = te.item()
+        e2e = {"value": round(world * P * m * n * ksteps / el / 1e9, 2), "unit": "GCUPS",
+               "h2d_bytes_per_step": world * P * (m + n), "d2h_bytes_per_step": world * P * 4,
+               "steps": ksteps, "timing": "host wall clock around the blocking C call "
+                                          "(pinned host buffers)"}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    # ---------------- parity sample against the oracle
+    import oracle
+    got = out.cpu().numpy()
+    rng = np.random.default_rng(seed)
+    idx = np.unique(np.concatenate([rng.choice(P, size=min(P, 2048), replace=False), [0, P - 1]]))
+    want = oracle.sw_batch(hq.numpy()[idx], ht.numpy()[idx], *CONSTS, score_bits=s)
+    parity = {"sampled_pairs": int(idx.size), "mismatches": int((got[idx] != want).sum())}
+
+    # ---------------- roofline of the sweep kernel (integer-logic pipe)
+    calls = max(1, phases["calls"])
+    sweep_ms = phases["swa_ms"] / calls
+    word_cells = (P + 31) // 32 * m * n
+    alg_ops = survey_ops_per_word_cell(s) * word_cells
+    achieved = alg_ops / (sweep_ms / 1e3) / 1e12
+    sm_max = clocks.get("sm_max_mhz") or 1965.0
+    peak = peak_alu_tops(sm_max)
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(f"C{args.config}")
+        except Exception:
+            traffic = None
+    roofline = {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 3),
+                "unit": "Tops/s (LOP3 lane-ops)", "frac": round(achieved / peak, 4),
+                "traffic": traffic, "kernel": "sw_sweep_kernel",
+                "kernel_ms_per_launch": round(sweep_ms, 4),
+                "alg_ops_per_word_cell": survey_ops_per_word_cell(s),
+                "evaluated_ops_per_word_cell": plan["ops_per_word_cell"],
+                "peak_basis": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM_CLK} LOP3 lanes/clk x "
+                              f"{sm_max:.0f} MHz (B300_MICROARCH alu rt=2/SMSP)",
+                "phase_ms_per_step": {k: round(v / calls, 4) for k, v in phases.items()
+                                      if k.endswith("_ms")}}
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        cpu = cpu_baseline(cfg)
+
+    line = {"metric": METRIC, "value": round(gcups, 2), "unit": "GCUPS", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(t_ms / args.steps, 4), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32 bit-sliced (s-bit scores)",
+            "data": "synthetic (seeded i.i.d. uniform DNA, SplitMix64)",
+            "config": {"workload": workload_name(args.config, cfg), "pairs_per_gpu": P,
+                       "m": m, "n": n, "score_bits": s, "parallelism": f"dp{world} (pair shards)",
+                       "l2": "inputs 320 MiB > 126 MB L2, plus a 256 MiB L2 flush between steps",
+                       "plan": plan},
+            "e2e": e2e, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,
+            "gpu_launches": 4 * args.steps * world, "parity": parity}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

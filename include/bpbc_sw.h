@@ -1,0 +1,191 @@
+/*
+ * bpbc_sw.h -- C ABI of the B200 (sm_100a) Bitwise Parallel Bulk Computation
+ * (BPBC) of the Smith-Waterman algorithm.
+ *
+ * Paper: T. Nishimura, J. L. Bordim, Y. Ito, K. Nakano, "Accelerating the
+ * Smith-Waterman Algorithm Using Bitwise Parallel Bulk Computation Technique
+ * on GPU", IPDPS Workshops 2017.  "P:Lnnn" cites line nnn of its text
+ * (PAPER.md); "Rk" cites reading k in DESIGN.md.
+ *
+ * Problem: num_pairs independent DNA pairs
+ * (X_k, Y_k), all with the same lengths m and n, stored wordwise (one byte
+ * per base, P:L350 / R15).  For each pair the library returns the maximum
+ * local-alignment score of the Smith-Waterman recurrence
+ *
+ *   d[i][j] = max(0, d[i-1][j] + gap, d[i][j-1] + gap,
+ *                 d[i-1][j-1] + (x_i == y_j ? match : mismatch)),
+ *   d[-1][.] = d[.][-1] = 0,  score = min(max_ij d[i][j], 2^score_bits - 1)
+ *
+ * (signed API constants: paper c1 = match, c2 = -mismatch, paper gap = -gap,
+ * R1; width cap R3).  Internally the pairs are bit-transposed 32 to a word
+ * (bit k = pair k) and every cell update runs as a Boolean circuit on
+ * bit-sliced s-bit scores, so one 32-bit logic op advances 32
+ * alignments.
+ *
+ * Base codes (R18): A = 0, T = 1, G = 2, C = 3 (the paper's A=00,
+ * T=01, G=10, C=11 with the H bit first).  Any byte > 3 is read as (c & 3)
+ * and raises the sticky BPBC_FLAG_BAD_BASE flag.
+ *
+ * Conventions for every function:
+ *   - returns a bpbc_status (0 = OK, < 0 error); never aborts, exits or
+ *     throws; no function writes to caller memory on an argument error;
+ *   - "device" pointers are CUDA device (or managed) memory of the ctx's
+ *     device; "host" pointers are host memory (pinned gives the fastest
+ *     copies);
+ *   - asynchronous functions only ENQUEUE work on `stream` (a cudaStream_t,
+ *     NULL = legacy default stream) and return; the caller keeps every
+ *     buffer alive until the stream has completed that work;
+ *   - a ctx is not thread-safe: use one ctx per device per host thread.
+ */
+#ifndef BPBC_SW_H
+#define BPBC_SW_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct bpbc_sw_ctx bpbc_sw_ctx;
+
+typedef enum {
+    BPBC_OK = 0,
+    BPBC_ERR_INVALID_ARG = -1, /* bad pointer / size / constant / workspace      */
+    BPBC_ERR_UNSUPPORTED = -2, /* valid but outside what this build supports     */
+    BPBC_ERR_CUDA = -3,        /* a CUDA call failed; text in bpbc_sw_last_error */
+    BPBC_ERR_OOM = -4,         /* device or host allocation failed               */
+    BPBC_ERR_BAD_BASE = -5     /* reported by bpbc_sw_check_flags               */
+} bpbc_status;
+
+/* Sticky device flags (bpbc_sw_get_error_flags). */
+#define BPBC_FLAG_BAD_BASE 0x1u /* a base code > 3 was packed (read as c & 3) */
+
+/* Supported ranges of this build. */
+#define BPBC_MIN_SCORE_BITS 4
+#define BPBC_MAX_SCORE_BITS 16
+#define BPBC_MAX_LEN (1 << 20) /* m, n <= 2^20 */
+
+/* Binds the context to `cuda_device`, creates its device flag word and
+ * queries the SM count.  No pair-sized allocation.  *out_ctx is set only on
+ * success. */
+int bpbc_sw_init(int cuda_device, bpbc_sw_ctx **out_ctx);
+
+/* Frees everything the ctx owns (its lazily grown workspace and host
+ * staging buffers).  Synchronizes the device first.  NULL is a no-op. */
+int bpbc_sw_destroy(bpbc_sw_ctx *ctx);
+
+/* Bytes of device workspace bpbc_sw_score_batch needs for these sizes:
+ * the bit-transposed planes 8 * ceil(P/32) * (m + n) bytes plus padding and
+ * the per-lane partial maxima (at most 2 KiB per 32-pair group per 256 query
+ * rows).  Pure host function. */
+int bpbc_sw_workspace_bytes(int64_t num_pairs, int32_t m, int32_t n, size_t *bytes);
+
+/*
+ * The hot path (Steps 2-4): pack (W2B) -> bit-sliced wavefront
+ * sweep with running max -> max over rows -> untranspose (B2W), all on the
+ * device, enqueued on `stream`.
+ *
+ * query       device, uint8 [num_pairs][m] row-major base codes (X_k).
+ * target      device, uint8 [num_pairs][n] row-major base codes (Y_k).
+ * num_pairs   >= 0; 0 is a no-op.  Need not be a multiple of 32.
+ * m, n        1 .. BPBC_MAX_LEN each; m > n is allowed (roles are swapped
+ *             internally; the score is symmetric, R17).  min(m, n) <= 256
+ *             in this build (else BPBC_ERR_UNSUPPORTED).
+ * match       >= 1                      (paper c1)
+ * mismatch    <= 0                      (paper -c2)
+ * gap         <= 0                      (paper -gap, linear per column)
+ * score_bits  s in [4, 16]: width of the bit-sliced score.  match,
+ *             -mismatch and -gap must each be <= 2^s - 1.  Results are
+ *             min(score, 2^s - 1) exactly (R3).
+ * out_scores  device, int32 [num_pairs].
+ * workspace   device scratch of >= bpbc_sw_workspace_bytes(...) bytes owned
+ *             by the caller, or NULL to use a ctx-owned buffer grown on
+ *             demand (allocation happens on the calling thread).
+ * stream      cudaStream_t to enqueue on.
+ *
+ * Errors (host-side, no device sync): INVALID_ARG for negative sizes, NULL
+ * pointers with num_pairs > 0, out-of-range constants or a too-small
+ * workspace; UNSUPPORTED for score_bits outside [4,16] or lengths beyond this
+ * build; CUDA if a launch fails.  Bad base codes cannot be seen without a
+ * sync: they set BPBC_FLAG_BAD_BASE.
+ */
+int bpbc_sw_score_batch(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8_t *target,
+                        int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                        int32_t mismatch, int32_t gap, int32_t score_bits,
+                        int32_t *out_scores, void *workspace, size_t workspace_bytes,
+                        void *stream);
+
+/*
+ * End-to-end variant with HOST buffers (the paper's Steps 1-5):
+ * copies the inputs host->device, runs the hot path and copies the scores
+ * device->host, chunked over pair ranges so copies of one chunk overlap the
+ * kernels of the previous one.  Blocking: returns when out_scores is
+ * written.  Uses ctx-owned device buffers.
+ *
+ * query, target  host, uint8 [num_pairs][m] / [num_pairs][n].
+ * out_scores     host, int32 [num_pairs].
+ * Other arguments as bpbc_sw_score_batch.
+ */
+int bpbc_sw_score_batch_host(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8_t *target,
+                             int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                             int32_t mismatch, int32_t gap, int32_t score_bits,
+                             int32_t *out_scores);
+
+/*
+ * W2B step alone: bit-transpose base codes into planes.
+ * codes   device, uint8 [num_pairs][len].
+ * planes  device, uint32 [ceil(num_pairs/32)][len][2]: [g][i][0] = X^H_i,
+ *         [g][i][1] = X^L_i of group g (bit k = pair 32g+k; pairs past
+ *         num_pairs read as code 0).
+ */
+int bpbc_sw_pack(bpbc_sw_ctx *ctx, const uint8_t *codes, int64_t num_pairs, int32_t len,
+                 uint32_t *planes, void *stream);
+
+/*
+ * Max-reduction + B2W step alone.
+ * partial    device, uint32 [num_groups][lanes][s]: lanes bit-sliced s-bit
+ *            values per 32-pair group (bit k of word b = bit b of pair k's
+ *            value).
+ * out        device, int32 [num_pairs] (num_pairs <= 32 * num_groups):
+ *            out[32g+k] = min(max over lanes of the value of pair k, cap).
+ * lanes in [1, 4096], s in [1, 16], cap >= 0.
+ */
+int bpbc_sw_untranspose(bpbc_sw_ctx *ctx, const uint32_t *partial, int64_t num_groups,
+                        int32_t lanes, int32_t s, int64_t num_pairs, int32_t cap,
+                        int32_t *out, void *stream);
+
+/* Synchronizes the ctx's device, returns the sticky flags in *flags (bit 0 =
+ * BPBC_FLAG_BAD_BASE) and clears them. */
+int bpbc_sw_get_error_flags(bpbc_sw_ctx *ctx, uint32_t *flags);
+
+/* Description of the last sweep dispatch (for benchmarks and tests):
+ * circuit 0 = exact offset circuit, 1 = saturating circuit; the score width
+ * actually evaluated; rows per lane R; lanes per 32-pair group L; concurrent
+ * group streams; and the bitwise-logic operations per word-cell of the
+ * evaluated circuit (hand count). Any pointer may be NULL. */
+int bpbc_sw_last_plan(bpbc_sw_ctx *ctx, int32_t *circuit, int32_t *width, int32_t *rows_per_lane,
+                      int32_t *lanes, int64_t *streams, int32_t *ops_per_word_cell);
+
+/* Per-phase device timing, the columns of the paper's Table IV (P:L384-413:
+ * W2B, SWA, B2W).  bpbc_sw_profile(ctx, 1) clears the accumulators and makes
+ * every following bpbc_sw_score_batch* call record CUDA events around its
+ * kernels on the call's stream; bpbc_sw_profile(ctx, 0) stops recording.
+ * bpbc_sw_profile_read synchronizes the recorded events and returns the
+ * summed milliseconds since the last read/enable:
+ *   ms[0] = W2B (both packs), ms[1] = SWA (sweep), ms[2] = B2W (extract),
+ *   ms[3] = their sum; *calls = number of calls recorded.  Then resets. */
+int bpbc_sw_profile(bpbc_sw_ctx *ctx, int enable);
+int bpbc_sw_profile_read(bpbc_sw_ctx *ctx, double ms[4], int64_t *calls);
+
+/* Static text for a status code. */
+const char *bpbc_sw_status_string(int status);
+
+/* Text of the last CUDA error seen by this ctx ("" if none). */
+const char *bpbc_sw_last_error(bpbc_sw_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* BPBC_SW_H */

@@ -1,0 +1,11 @@
+"""B200 (sm_100a) Bitwise Parallel Bulk Computation of the Smith-Waterman
+algorithm (Nishimura, Bordim, Ito, Nakano, IPDPSW 2017).
+
+Public API (same names as the C ABI in include/bpbc_sw.h):
+  score_batch, score_batch_host, pack, untranspose, workspace_bytes,
+  get_error_flags, last_plan; multi-GPU: parallel.score_sharded.
+"""
+from ._lib import BPBCError, LIB_PATH  # noqa: F401
+from .api import (default_score_bits, destroy_all, get_error_flags, last_plan, pack,  # noqa: F401
+                  profile, profile_read, score_batch, score_batch_host, untranspose,
+                  workspace_bytes)

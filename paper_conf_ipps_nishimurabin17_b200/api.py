@@ -1,0 +1,165 @@
+"""Python binding of the BPBC Smith-Waterman C ABI (include/bpbc_sw.h).
+
+Same names as the C entry points; torch is used for device memory and
+streams only.  Every step of the path (pack, sweep, max reduction,
+untranspose) runs in the CUDA kernels of libbpbc_sw.so.
+"""
+from __future__ import annotations
+
+import ctypes
+import threading
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import check
+
+_ctx_lock = threading.Lock()
+_ctxs: dict[int, ctypes.c_void_p] = {}
+
+
+def _ctx(device: int) -> ctypes.c_void_p:
+    with _ctx_lock:
+        c = _ctxs.get(device)
+        if c is None:
+            c = ctypes.c_void_p()
+            check(_lib.load().bpbc_sw_init(device, ctypes.byref(c)))
+            _ctxs[device] = c
+        return c
+
+
+def destroy_all() -> None:
+    with _ctx_lock:
+        for c in _ctxs.values():
+            _lib.load().bpbc_sw_destroy(c)
+        _ctxs.clear()
+
+
+def default_score_bits(match: int, m: int, n: int) -> int:
+    """s = bit_length(match * min(m, n)) (reading R2), in [4, 16]."""
+    return min(16, max(4, (match * min(m, n)).bit_length()))
+
+
+def _stream_ptr(stream, device) -> int:
+    if stream is None:
+        stream = torch.cuda.current_stream(device)
+    return stream.cuda_stream
+
+
+def workspace_bytes(num_pairs: int, m: int, n: int) -> int:
+    v = ctypes.c_size_t()
+    check(_lib.load().bpbc_sw_workspace_bytes(num_pairs, m, n, ctypes.byref(v)))
+    return v.value
+
+
+def score_batch(query: torch.Tensor, target: torch.Tensor, match: int = 2, mismatch: int = -1,
+                gap: int = -1, score_bits: int | None = None, out: torch.Tensor | None = None,
+                workspace: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """bpbc_sw_score_batch on CUDA tensors query uint8 [P, m], target uint8 [P, n].
+
+    Returns int32 [P] = min(max local score, 2^score_bits - 1), enqueued on
+    ``stream`` (default: torch's current stream of the tensors' device)."""
+    if not (query.is_cuda and target.is_cuda):
+        raise ValueError("score_batch needs CUDA tensors (use score_batch_host for host arrays)")
+    if query.dtype != torch.uint8 or target.dtype != torch.uint8:
+        raise TypeError("query/target must be uint8 base codes")
+    if query.dim() != 2 or target.dim() != 2 or query.shape[0] != target.shape[0]:
+        raise ValueError("query [P, m] and target [P, n] expected")
+    query, target = query.contiguous(), target.contiguous()
+    P, m = query.shape
+    n = target.shape[1]
+    dev = query.device.index if query.device.index is not None else torch.cuda.current_device()
+    if score_bits is None:
+        score_bits = default_score_bits(match, m, n)
+    if out is None:
+        out = torch.empty(P, dtype=torch.int32, device=query.device)
+    ws_ptr, ws_bytes = None, 0
+    if workspace is not None:
+        ws_ptr, ws_bytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
+    ctx = _ctx(dev)
+    check(_lib.load().bpbc_sw_score_batch(ctx, query.data_ptr(), target.data_ptr(), P, m, n, match,
+                                          mismatch, gap, score_bits, out.data_ptr(), ws_ptr,
+                                          ws_bytes, _stream_ptr(stream, query.device)), ctx)
+    return out
+
+
+def score_batch_host(query: np.ndarray, target: np.ndarray, match: int = 2, mismatch: int = -1,
+                     gap: int = -1, score_bits: int | None = None, device: int = 0,
+                     out: np.ndarray | None = None) -> np.ndarray:
+    """bpbc_sw_score_batch_host: host arrays in, host int32 scores out (blocking).
+    ``query``/``target`` may be numpy views of pinned torch tensors."""
+    query = np.ascontiguousarray(query, dtype=np.uint8)
+    target = np.ascontiguousarray(target, dtype=np.uint8)
+    P, m = query.shape
+    n = target.shape[1]
+    if score_bits is None:
+        score_bits = default_score_bits(match, m, n)
+    if out is None:
+        out = np.empty(P, dtype=np.int32)
+    ctx = _ctx(device)
+    check(_lib.load().bpbc_sw_score_batch_host(ctx, query.ctypes.data, target.ctypes.data, P, m, n,
+                                               match, mismatch, gap, score_bits, out.ctypes.data),
+          ctx)
+    return out
+
+
+def pack(codes: torch.Tensor, stream=None) -> torch.Tensor:
+    """bpbc_sw_pack: uint8 [P, len] -> uint32 [ceil(P/32), len, 2] bit planes (H, L)."""
+    codes = codes.contiguous()
+    P, ln = codes.shape
+    G = (P + 31) // 32
+    planes = torch.empty((G, ln, 2), dtype=torch.int32, device=codes.device)
+    dev = codes.device.index or 0
+    ctx = _ctx(dev)
+    check(_lib.load().bpbc_sw_pack(ctx, codes.data_ptr(), P, ln, planes.data_ptr(),
+                                   _stream_ptr(stream, codes.device)), ctx)
+    return planes
+
+
+def untranspose(partial: torch.Tensor, num_pairs: int, cap: int, stream=None) -> torch.Tensor:
+    """bpbc_sw_untranspose: uint32 [G, lanes, s] bit-sliced partial maxima ->
+    int32 [num_pairs] = min(max over lanes, cap)."""
+    partial = partial.contiguous()
+    G, lanes, s = partial.shape
+    out = torch.empty(num_pairs, dtype=torch.int32, device=partial.device)
+    dev = partial.device.index or 0
+    ctx = _ctx(dev)
+    check(_lib.load().bpbc_sw_untranspose(ctx, partial.data_ptr(), G, lanes, s, num_pairs, cap,
+                                          out.data_ptr(), _stream_ptr(stream, partial.device)), ctx)
+    return out
+
+
+def get_error_flags(device: int = 0) -> int:
+    v = ctypes.c_uint32()
+    ctx = _ctx(device)
+    check(_lib.load().bpbc_sw_get_error_flags(ctx, ctypes.byref(v)), ctx)
+    return v.value
+
+
+def last_plan(device: int = 0) -> dict:
+    """Circuit / width / tiling of the last sweep dispatched on ``device``."""
+    c, w, r, l, o = (ctypes.c_int32() for _ in range(5))
+    s = ctypes.c_int64()
+    check(_lib.load().bpbc_sw_last_plan(_ctx(device), ctypes.byref(c), ctypes.byref(w),
+                                        ctypes.byref(r), ctypes.byref(l), ctypes.byref(s),
+                                        ctypes.byref(o)))
+    return {"circuit": ["exact", "saturating"][c.value] if c.value >= 0 else None,
+            "width": w.value, "rows_per_lane": r.value, "lanes": l.value,
+            "streams": s.value, "ops_per_word_cell": o.value}
+
+
+def profile(enable: bool, device: int = 0) -> None:
+    """bpbc_sw_profile: start (clearing) / stop per-phase event recording."""
+    check(_lib.load().bpbc_sw_profile(_ctx(device), int(bool(enable))))
+
+
+def profile_read(device: int = 0) -> dict:
+    """bpbc_sw_profile_read: summed ms per phase (Table IV columns W2B, SWA,
+    B2W) over the calls recorded since the last read; resets."""
+    ms = (ctypes.c_double * 4)()
+    calls = ctypes.c_int64()
+    ctx = _ctx(device)
+    check(_lib.load().bpbc_sw_profile_read(ctx, ms, ctypes.byref(calls)), ctx)
+    return {"w2b_ms": ms[0], "swa_ms": ms[1], "b2w_ms": ms[2], "total_ms": ms[3],
+            "calls": calls.value}

@@ -1,0 +1,77 @@
+// bpbc_internal.cuh -- shared layout and launch declarations of the CUDA path.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "bpbc_sw.h"
+#include "circuit.cuh"
+
+namespace bpbc {
+
+// Planes buffers carry padding so the sweep never bounds-checks its loads:
+// the Y stream of a warp is read at virtual column J = tau - lane, which runs
+// up to L columns before its first group and up to n + L columns past its
+// last.
+constexpr int64_t kYFrontPad = 64;   // uint2 words before Y plane 0
+constexpr int64_t kXBackPad = 512;   // uint2 words after the last X group
+constexpr int64_t kYBackPadExtra = 128;
+
+enum Circuit : int { kExact = 0, kSat = 1 };
+enum Consts : int { kC211 = 0, kCRun = 1 };
+constexpr int kNumVariants = 8;  // circuit x consts x padded-rows
+constexpr int variant_index(int circuit, int consts, bool pad) {
+  return (circuit * 2 + consts) * 2 + (pad ? 1 : 0);
+}
+
+// Arguments of the sweep kernel (one struct, passed by value).
+struct SweepArgs {
+  const uint2* Xp;   // [G][m] (+kXBackPad) query planes {H, L}
+  const uint2* Yp;   // points at Y plane 0 of group 0: [G][n], padded both sides
+  uint32_t* Mpart;   // [G][L][S] per-lane partial maxima (bit-sliced)
+  int64_t G;         // 32-pair groups
+  int m, n;          // query rows (m <= L*R), target columns
+  int64_t streams;   // number of group streams (one per L lanes)
+  int64_t base;      // groups per stream: base or base+1
+  int64_t rem;       //   (the first rem streams get base+1)
+  int64_t steps;     // wavefront steps = (base + (rem>0)) * n + L
+};
+
+typedef void (*SweepLaunchFn)(const SweepArgs&, const KRun&, int grid, int block,
+                              cudaStream_t stream);
+
+// Registry of compiled sweep kernels: [variant_index][rl][S - 4].
+constexpr int kNumRL = 4;  // (R, L) in {(2,16), (4,16), (4,32), (8,32)}
+constexpr int kRLR[kNumRL] = {2, 4, 4, 8};
+constexpr int kRLL[kNumRL] = {16, 16, 32, 32};
+struct SweepEntry {
+  SweepLaunchFn launch;
+  const void* func;  // kernel pointer for occupancy queries
+};
+SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
+
+// Registration hooks, one per score width (sweep.cu compiled once per S).
+#define BPBC_DECLARE_REG(S) void register_sweep_s##S(SweepEntry (*tab)[kNumRL][13]);
+BPBC_DECLARE_REG(4)
+BPBC_DECLARE_REG(5)
+BPBC_DECLARE_REG(6)
+BPBC_DECLARE_REG(7)
+BPBC_DECLARE_REG(8)
+BPBC_DECLARE_REG(9)
+BPBC_DECLARE_REG(10)
+BPBC_DECLARE_REG(11)
+BPBC_DECLARE_REG(12)
+BPBC_DECLARE_REG(13)
+BPBC_DECLARE_REG(14)
+BPBC_DECLARE_REG(15)
+BPBC_DECLARE_REG(16)
+#undef BPBC_DECLARE_REG
+
+// pack.cu
+cudaError_t launch_pack(const uint8_t* codes, int64_t num_pairs, int len, uint2* planes,
+                        uint32_t* flags, int num_sms, cudaStream_t stream);
+// extract.cu
+cudaError_t launch_extract(const uint32_t* partial, int64_t num_groups, int lanes, int s,
+                           int64_t num_pairs, int32_t cap, int32_t* out, int num_sms,
+                           cudaStream_t stream);
+
+}  // namespace bpbc

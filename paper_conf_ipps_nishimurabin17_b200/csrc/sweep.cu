@@ -1,0 +1,201 @@
+// sweep.cu -- the BPBC Smith-Waterman cell sweep (the hot loop), sm_100a.
+//
+// Compiled once per score width S (-DBPBC_S=S) so the 13 widths build in
+// parallel; each object registers its kernels in the dispatch table.
+//
+// What it computes ("BPBC parallel for SWA", and the per-thread
+// program of P:L364-372): for every 32-pair group, the bit-sliced score
+// tables D^l[i][j] cell by cell along anti-diagonals t = i + j
+// (R7), keeping the running maximum R_{k,i} per row and
+// writing it per lane for the max-reduction + B2W step (extract.cu).
+//
+// B200 design, not the paper's TITAN X one:
+//   * one 32-pair group per L lanes (L = 16 or 32; 32/L groups per warp);
+//     lane l owns query rows [l*R, l*R + R) and keeps their current scores
+//     (R*S planes), its query bases (2R words) and its running max (S planes)
+//     in registers for the whole group -- no shared memory on the path
+//     (the paper hands rows over through shared memory);
+//   * wavefront skew across lanes: at step tau lane l works on column
+//     J = tau - l; the bottom-row scores move to lane l+1 with S
+//     __shfl_up_sync per step (the paper names shuffles as the option);
+//   * persistent streaming: each L-lane segment walks a contiguous range of
+//     groups back to back as one virtual target of length Gs*n, so the
+//     pipeline fill/drain (L-1 steps, the paper's (m-1)/(n+m-1) idle share)
+//     is paid once per stream, not per group;
+//   * the group switch of a lane (its column J hits a multiple of n) resets
+//     its state in a short divergent branch taken once per group per lane;
+//   * the cell is a fixed LOP3 circuit (circuit.cuh): no branch on data.
+#include "bpbc_internal.cuh"
+
+#ifndef BPBC_S
+#error "compile with -DBPBC_S=<score width>"
+#endif
+
+namespace bpbc {
+namespace {
+
+__device__ __forceinline__ uint32_t opaque(uint32_t v) {
+  uint32_t r;
+  asm volatile("mov.b32 %0, %1;" : "=r"(r) : "r"(v));
+  return r;
+}
+__device__ __forceinline__ uint32_t mul_lo(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm("mul.lo.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+
+template <int S, int R, int L, int CIRC, bool PAD, class K>
+__global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const K k) {
+  constexpr int SEGS = 32 / L;
+  const int lane = threadIdx.x & 31;
+  const int sl = lane & (L - 1);
+  const int64_t warp = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  if (warp * SEGS >= a.streams) return;  // uniform per warp
+  const int64_t stream = warp * SEGS + lane / L;
+
+  int64_t Gs = 0, gb = 0;
+  if (stream < a.streams) {
+    Gs = a.base + (stream < a.rem ? 1 : 0);
+    gb = stream * a.base + (stream < a.rem ? stream : a.rem);
+  }
+  // 1 for lanes that receive a real "up" row from the lane above, 0 for the
+  // first lane of a segment (border d[-1][j] = 0).  Applied with an
+  // integer multiply so it issues on the FMA pipe, not the logic pipe.
+  // (volatile moves keep these opaque: the compiler may neither turn the
+  // multiply into a logic-pipe select nor rematerialise the masks per step)
+  const uint32_t nz = opaque(sl != 0 ? 1u : 0u);
+
+  // kill[r] = all ones for padded rows (row >= m): their cells output 0.
+  uint32_t kill[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) kill[r] = PAD ? opaque((sl * R + r >= a.m) ? 0xFFFFFFFFu : 0u) : 0u;
+
+  uint32_t H[R][S];   // scores of my rows at the previous column (left)
+  uint32_t dtop[S];   // up-row score at the previous column (diag of row 0)
+  uint32_t M[S];      // running max of my rows
+#pragma unroll
+  for (int i = 0; i < S; ++i) {
+    dtop[i] = 0;
+    M[i] = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) H[r][i] = 0;
+  }
+  uint32_t xh[R], xl[R], nxh[R], nxl[R];
+  {
+    const uint2* xp = a.Xp + (gb < a.G ? gb : a.G - 1) * a.m + sl * R;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const uint2 v = __ldg(xp + r);
+      nxh[r] = v.x;
+      nxl[r] = v.y;
+      xh[r] = xl[r] = 0;
+    }
+  }
+  const uint2* yp = a.Yp + gb * a.n - sl;
+  int cnt = sl;      // steps until my next group starts (J % n == 0)
+  int64_t gi = -1;   // my current group within the stream
+
+  for (int64_t tau = 0; tau < a.steps; ++tau) {
+    uint32_t up[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
+
+    if (cnt == 0) {  // column 0 of my next group (divergent, once per group)
+      if (gi >= 0 && gi < Gs) {
+        uint32_t* dst = a.Mpart + ((gb + gi) * L + sl) * S;
+#pragma unroll
+        for (int i = 0; i < S; ++i) dst[i] = M[i];
+      }
+      ++gi;
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        M[i] = 0;
+        dtop[i] = 0;
+#pragma unroll
+        for (int r = 0; r < R; ++r) H[r][i] = 0;
+      }
+      int64_t nxt = gb + gi + 1;
+      nxt = nxt < a.G ? nxt : a.G - 1;
+      const uint2* xp = a.Xp + nxt * a.m + sl * R;
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        xh[r] = nxh[r];
+        xl[r] = nxl[r];
+        const uint2 v = __ldg(xp + r);
+        nxh[r] = v.x;
+        nxl[r] = v.y;
+      }
+      cnt = a.n;
+    }
+    --cnt;
+
+    const uint2 y = __ldg(yp + tau);
+    uint32_t dg[S], u[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      dg[i] = dtop[i];
+      u[i] = up[i];
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      uint32_t hn[S];
+      if constexpr (CIRC == kExact) {
+        cell_exact<S, K, PAD>(u, H[r], dg, xh[r], xl[r], y.x, y.y, kill[r], hn);
+        runmax<S, false>(M, hn, 0u);
+      } else {
+        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, k);
+        runmax<S, PAD>(M, hn, kill[r]);
+      }
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        dg[i] = H[r][i];
+        H[r][i] = hn[i];
+        u[i] = hn[i];
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < S; ++i) dtop[i] = up[i];
+  }
+}
+
+template <int S, int R, int L, int CIRC, bool PAD, class K>
+void launch_sweep(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
+  if constexpr (K::kFixed) {
+    sw_sweep_kernel<S, R, L, CIRC, PAD, K><<<grid, block, 0, st>>>(a, K{});
+  } else {
+    sw_sweep_kernel<S, R, L, CIRC, PAD, KRun><<<grid, block, 0, st>>>(a, kr);
+  }
+}
+
+template <int S, int RL, bool PAD>
+void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
+  constexpr int R = kRLR[RL], L = kRLL[RL];
+  using K211 = KFix<2, 1, 1>;
+  tab[variant_index(kExact, kC211, PAD)][RL][S - 4] = {
+      &launch_sweep<S, R, L, kExact, PAD, K211>,
+      (const void*)&sw_sweep_kernel<S, R, L, kExact, PAD, K211>};
+  tab[variant_index(kSat, kC211, PAD)][RL][S - 4] = {
+      &launch_sweep<S, R, L, kSat, PAD, K211>,
+      (const void*)&sw_sweep_kernel<S, R, L, kSat, PAD, K211>};
+  tab[variant_index(kSat, kCRun, PAD)][RL][S - 4] = {
+      &launch_sweep<S, R, L, kSat, PAD, KRun>,
+      (const void*)&sw_sweep_kernel<S, R, L, kSat, PAD, KRun>};
+}
+
+}  // namespace
+
+#define BPBC_CAT2(a, b) a##b
+#define BPBC_CAT(a, b) BPBC_CAT2(a, b)
+void BPBC_CAT(register_sweep_s, BPBC_S)(SweepEntry (*tab)[kNumRL][13]) {
+  reg_rl<BPBC_S, 0, false>(tab);
+  reg_rl<BPBC_S, 1, false>(tab);
+  reg_rl<BPBC_S, 2, false>(tab);
+  reg_rl<BPBC_S, 3, false>(tab);
+  reg_rl<BPBC_S, 0, true>(tab);
+  reg_rl<BPBC_S, 1, true>(tab);
+  reg_rl<BPBC_S, 2, true>(tab);
+  reg_rl<BPBC_S, 3, true>(tab);
+}
+
+}  // namespace bpbc

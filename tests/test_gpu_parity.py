@@ -1,0 +1,246 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle, element by
+element on the same seeded inputs (bit-exact, integer results).
+
+Small/medium sizes are checked in full; BASELINE.json's full sizes run in the
+launch configuration bench.py times and are checked on a seeded sample of
+pairs (the oracle scores each sampled pair on its own).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+import paper_conf_ipps_nishimurabin17_b200 as bpbc
+from paper_conf_ipps_nishimurabin17_b200 import _lib
+
+pytestmark = pytest.mark.gpu
+
+DEV = "cuda:0"
+
+
+def run(q, t, match=2, mismatch=-1, gap=-1, s=None):
+    dq = torch.from_numpy(np.ascontiguousarray(q)).to(DEV)
+    dt = torch.from_numpy(np.ascontiguousarray(t)).to(DEV)
+    out = bpbc.score_batch(dq, dt, match, mismatch, gap, score_bits=s)
+    return out.cpu().numpy()
+
+
+def check_full(q, t, match=2, mismatch=-1, gap=-1, s=None):
+    m, n = q.shape[1], t.shape[1]
+    if s is None:
+        s = bpbc.default_score_bits(match, m, n)
+    got = run(q, t, match, mismatch, gap, s)
+    want = oracle.sw_batch(q, t, match, mismatch, gap, score_bits=s)
+    bad = np.nonzero(got != want)[0]
+    assert bad.size == 0, (f"{bad.size}/{len(want)} mismatches (m={m}, n={n}, s={s}, "
+                           f"consts={match},{mismatch},{gap}, plan={bpbc.last_plan(0)}); "
+                           f"first pair {bad[0]}: got {got[bad[0]]} want {want[bad[0]]}")
+    return got
+
+
+# ---------------------------------------------------------------- configs
+
+
+def test_c1_full():
+    """BASELINE config 1: 1024 pairs, m = n = 64, +2/-1/-1, 8-bit slices."""
+    q, t = synth.gen_pairs(synth.seed_for_config(1), 1024, 64, 64, planted=True)
+    got = check_full(q, t, s=8)
+    assert got.max() == 128  # planted exact copies reach m * match
+    assert bpbc.last_plan(0)["circuit"] == "exact"
+
+
+@pytest.mark.parametrize("P,m,n,s", [(16384, 128, 128, 9), (4096, 256, 256, 10),
+                                     (4096, 64, 1024, 8), (8192, 32, 32, 6), (8192, 64, 64, 7)])
+def test_config_shapes_full(P, m, n, s):
+    q, t = synth.gen_pairs(synth.seed_for_config(10) + m + n, P, m, n, planted=True)
+    check_full(q, t, s=s)
+
+
+def _sampled(cfg_id, P, m, n, s, sample=8192):
+    q, t = synth.gen_pairs(synth.seed_for_config(cfg_id), P, m, n, planted=True)
+    got = run(q, t, 2, -1, -1, s)
+    rng = np.random.default_rng(cfg_id)
+    idx = np.sort(rng.choice(P, size=sample, replace=False))
+    idx = np.concatenate([idx, [0, P - 1]])
+    want = oracle.sw_batch(q[idx], t[idx], 2, -1, -1, score_bits=s)
+    np.testing.assert_array_equal(got[idx], want)
+    # properties at any size: 0 <= score <= min(2*min(m,n), 2^s-1)
+    assert got.min() >= 0 and got.max() <= min(2 * min(m, n), 2 ** s - 1)
+
+
+def test_c2_full_size_sampled():
+    """BASELINE config 2 at full size (2^20 pairs, m=n=128, s=9)."""
+    _sampled(2, 1 << 20, 128, 128, 9)
+
+
+def test_c4_full_size_sampled():
+    """BASELINE config 4 at full size (2^20 pairs, m=64, n=1024, s=8)."""
+    _sampled(4, 1 << 20, 64, 1024, 8, sample=4096)
+
+
+def test_c3_full_size_sampled():
+    """BASELINE config 3 per-GPU shard at full size (2^22 pairs, m=n=256, s=10)."""
+    _sampled(3, 1 << 22, 256, 256, 10, sample=4096)
+
+
+# ---------------------------------------------------------------- edge cases
+
+
+@pytest.mark.parametrize("P", [1, 31, 32, 33, 95, 1000])
+def test_ragged_pair_counts(P):
+    q, t = synth.gen_pairs(77 + P, P, 40, 56, planted=True)
+    check_full(q, t)
+
+
+@pytest.mark.parametrize("m,n", [(1, 1), (1, 9), (9, 1), (3, 300), (17, 5), (33, 33), (63, 65),
+                                 (100, 100), (129, 130), (200, 64), (255, 255), (256, 256),
+                                 (256, 1000), (64, 2000)])
+def test_lengths(m, n):
+    q, t = synth.gen_pairs(5000 + m * 131 + n, 200, m, n, planted=True)
+    check_full(q, t)
+
+
+@pytest.mark.parametrize("s", list(range(4, 17)))
+def test_every_width_spec_consts(s):
+    q, t = synth.gen_pairs(600 + s, 512, 48, 80, planted=True)
+    check_full(q, t, s=s)
+
+
+@pytest.mark.parametrize("consts", [(1, -1, -1), (3, -2, -1), (1, 0, 0), (2, 0, -1), (5, -3, -4),
+                                    (2, -3, -2), (1, -1, 0), (4, -1, -2)])
+@pytest.mark.parametrize("s", [5, 8, 12])
+def test_runtime_constants(consts, s):
+    q, t = synth.gen_pairs(700 + s, 300, 37, 61, planted=True)
+    c1, mm, g = consts
+    if max(c1, -mm, -g) > 2 ** s - 1:
+        pytest.skip("constants must fit")
+    check_full(q, t, c1, mm, g, s)
+
+
+@pytest.mark.parametrize("m", [32, 64, 128, 256])
+@pytest.mark.parametrize("s", [6, 7, 8, 9, 10, 11, 12])
+def test_c5_width_sweep_saturation(m, s):
+    """C5-shaped: the width sweep saturates most pairs at small s (R3)."""
+    q, t = synth.gen_pairs(synth.seed_for_config(5) + m, 2048, m, m, planted=True)
+    got = check_full(q, t, s=s)
+    exact = oracle.sw_batch(q, t, 2, -1, -1)
+    np.testing.assert_array_equal(got, np.minimum(exact, 2 ** s - 1))
+
+
+def test_empty_batch_is_noop():
+    q = torch.empty((0, 10), dtype=torch.uint8, device=DEV)
+    t = torch.empty((0, 12), dtype=torch.uint8, device=DEV)
+    out = bpbc.score_batch(q, t)
+    assert out.numel() == 0
+
+
+def test_errors():
+    q = torch.zeros((4, 10), dtype=torch.uint8, device=DEV)
+    t = torch.zeros((4, 300), dtype=torch.uint8, device=DEV)
+    with pytest.raises(bpbc.BPBCError) as ei:
+        bpbc.score_batch(q, t, 2, -1, -1, score_bits=3)
+    assert ei.value.status == _lib.BPBC_ERR_UNSUPPORTED
+    with pytest.raises(bpbc.BPBCError) as ei:
+        bpbc.score_batch(q, t, 0, -1, -1, score_bits=8)
+    assert ei.value.status == _lib.BPBC_ERR_INVALID_ARG
+    with pytest.raises(bpbc.BPBCError) as ei:
+        bpbc.score_batch(q, t, 2, 1, -1, score_bits=8)
+    assert ei.value.status == _lib.BPBC_ERR_INVALID_ARG
+    with pytest.raises(bpbc.BPBCError) as ei:
+        bpbc.score_batch(q, t, 2, -1, -20, score_bits=4)
+    assert ei.value.status == _lib.BPBC_ERR_INVALID_ARG
+    big = torch.zeros((4, 300), dtype=torch.uint8, device=DEV)
+    with pytest.raises(bpbc.BPBCError) as ei:
+        bpbc.score_batch(big, big)
+    assert ei.value.status == _lib.BPBC_ERR_UNSUPPORTED
+    ws = torch.empty(16, dtype=torch.uint8, device=DEV)
+    with pytest.raises(bpbc.BPBCError) as ei:
+        bpbc.score_batch(q, q, workspace=ws)
+    assert ei.value.status == _lib.BPBC_ERR_INVALID_ARG
+
+
+def test_caller_workspace_and_stream():
+    q, t = synth.gen_pairs(31337, 777, 50, 70, planted=True)
+    ws = torch.empty(bpbc.workspace_bytes(777, 50, 70), dtype=torch.uint8, device=DEV)
+    st = torch.cuda.Stream(device=DEV)
+    dq = torch.from_numpy(q).to(DEV)
+    dt = torch.from_numpy(t).to(DEV)
+    torch.cuda.synchronize()
+    with torch.cuda.stream(st):
+        out = bpbc.score_batch(dq, dt, workspace=ws, stream=st)
+    st.synchronize()
+    np.testing.assert_array_equal(out.cpu().numpy(),
+                                  oracle.sw_batch(q, t, 2, -1, -1, score_bits=8))
+
+
+def test_bad_base_flag():
+    q, t = synth.gen_pairs(9, 64, 20, 20)
+    bpbc.get_error_flags(0)  # clear
+    q2 = q.copy()
+    q2[5, 3] = 7  # not a base code: read as 7 & 3 = 3, flagged
+    got = run(q2, t, s=8)
+    assert bpbc.get_error_flags(0) & _lib.BPBC_FLAG_BAD_BASE
+    np.testing.assert_array_equal(got, oracle.sw_batch(q2 & 3, t, 2, -1, -1, score_bits=8))
+    run(q, t, s=8)
+    assert bpbc.get_error_flags(0) == 0
+
+
+def test_host_buffer_path():
+    q, t = synth.gen_pairs(4242, 3000, 64, 96, planted=True)
+    got = bpbc.score_batch_host(q, t, 2, -1, -1, 8)
+    np.testing.assert_array_equal(got, oracle.sw_batch(q, t, 2, -1, -1, score_bits=8))
+
+
+def test_deterministic_and_input_independent_plan():
+    q, t = synth.gen_pairs(11, 4096, 128, 128)
+    a = run(q, t, s=9)
+    b = run(q, t, s=9)
+    np.testing.assert_array_equal(a, b)
+
+
+# ---------------------------------------------------------------- single steps
+
+
+@pytest.mark.parametrize("P,ln", [(4, 5), (1, 1), (33, 31), (100, 64), (64, 100), (1000, 129),
+                                  (257, 1024)])
+def test_pack_kernel_matches_definition(P, ln):
+    rng = np.random.default_rng(P * 1000 + ln)
+    codes = rng.integers(0, 4, size=(P, ln), dtype=np.uint8)
+    planes = bpbc.pack(torch.from_numpy(codes).to(DEV)).cpu().numpy().view(np.uint32)
+    np.testing.assert_array_equal(planes, oracle.pack_planes(codes))
+
+
+def test_pack_kernel_paper_example():
+    """The 4-pair planes of P:L65-79 through the CUDA pack kernel."""
+    xs = np.stack([synth.encode(s) for s in ["ATCGA", "TCGAC", "AAAAA", "TTTTT"]])
+    ys = np.stack([synth.encode(s) for s in ["AATCGACA"] * 2 + ["AAAAAAAA", "AATTTTTT"]])
+    px = bpbc.pack(torch.from_numpy(xs).to(DEV)).cpu().numpy().view(np.uint32)
+    py = bpbc.pack(torch.from_numpy(ys).to(DEV)).cpu().numpy().view(np.uint32)
+    assert [int(w) for w in px[0, :, 0]] == [0b0000, 0b0010, 0b0011, 0b0001, 0b0010]
+    assert [int(w) for w in px[0, :, 1]] == [0b1010, 0b1011, 0b1001, 0b1000, 0b1010]
+    assert [int(w) for w in py[0, :, 0]] == [0, 0, 0, 0b0011, 0b0011, 0, 0b0011, 0]
+    assert [int(w) for w in py[0, :, 1]] == [0, 0, 0b1011, 0b1011, 0b1000, 0b1000, 0b1011, 0b1000]
+
+
+@pytest.mark.parametrize("lanes,s", [(1, 4), (16, 9), (32, 10), (33, 16), (64, 8), (100, 12)])
+def test_untranspose_kernel(lanes, s):
+    rng = np.random.default_rng(lanes * 100 + s)
+    G = 37
+    vals = rng.integers(0, 2 ** s, size=(G, lanes, 32))
+    partial = np.zeros((G, lanes, s), dtype=np.uint32)
+    for b in range(s):
+        partial[:, :, b] = (((vals >> b) & 1).astype(np.uint64) << np.arange(32, dtype=np.uint64)
+                            ).sum(axis=2).astype(np.uint32)
+    cap = 2 ** s - 1 - 3
+    P = G * 32 - 5
+    got = bpbc.untranspose(torch.from_numpy(partial.view(np.int32)).to(DEV), P, cap).cpu().numpy()
+    want = np.minimum(vals.max(axis=1).reshape(-1), cap)[:P]
+    np.testing.assert_array_equal(got, want)
+    # the definition in the oracle agrees on the reduced planes
+    red = np.zeros((G, s), dtype=np.uint32)
+    mx = vals.max(axis=1)
+    for b in range(s):
+        red[:, b] = (((mx >> b) & 1).astype(np.uint64) << np.arange(32, dtype=np.uint64)
+                     ).sum(axis=1).astype(np.uint32)
+    np.testing.assert_array_equal(np.minimum(oracle.untranspose(red), cap)[:P], want)
