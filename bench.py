@@ -310,7 +310,9 @@ def main():
     calls = max(1, phases["calls"])
     sweep_ms = phases["swa_ms"] / calls
     word_cells = (P + 31) // 32 * m * n
-    alg_ops = survey_ops_per_word_cell(s) * word_cells
+    # algorithmic LOP3 per word-cell = hand count of the circuit the plan
+    # evaluates; SURVEY's 11s+2 is printed beside it
+    alg_ops = plan["ops_per_word_cell"] * word_cells
     achieved = alg_ops / (sweep_ms / 1e3) / 1e12
     sm_max = clocks.get("sm_max_mhz") or 1965.0
     peak = peak_alu_tops(sm_max)
@@ -318,15 +320,16 @@ def main():
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get(f"C{args.config}")
+            traffic = json.load(open(tp)).get(f"C{args.config}", {}).get("sweep_dram_bytes")
         except Exception:
             traffic = None
     roofline = {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 3),
                 "unit": "Tops/s (LOP3 lane-ops)", "frac": round(achieved / peak, 4),
                 "traffic": traffic, "kernel": "sw_sweep_kernel",
                 "kernel_ms_per_launch": round(sweep_ms, 4),
-                "alg_ops_per_word_cell": survey_ops_per_word_cell(s),
-                "evaluated_ops_per_word_cell": plan["ops_per_word_cell"],
+                "alg_ops_per_word_cell": plan["ops_per_word_cell"],
+                "alg_ops_per_word_cell_survey": survey_ops_per_word_cell(s),
+                "word_cells_per_launch": word_cells,
                 "peak_basis": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM_CLK} LOP3 lanes/clk x "
                               f"{sm_max:.0f} MHz (B300_MICROARCH alu rt=2/SMSP)",
                 "phase_ms_per_step": {k: round(v / calls, 4) for k, v in phases.items()
