@@ -9,3 +9,5 @@ from ._lib import BPBCError, LIB_PATH  # noqa: F401
 from .api import (default_score_bits, destroy_all, get_error_flags, last_plan, pack,  # noqa: F401
                   profile, profile_read, score_batch, score_batch_host, untranspose,
                   workspace_bytes)
+from .parallel import (gather_scores, score_multi_device, score_sharded, shard_range,  # noqa: F401
+                       shard_ranges)

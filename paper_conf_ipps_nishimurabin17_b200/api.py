@@ -16,16 +16,19 @@ from . import _lib
 from ._lib import check
 
 _ctx_lock = threading.Lock()
-_ctxs: dict[int, ctypes.c_void_p] = {}
+_ctxs: dict[tuple[int, int], ctypes.c_void_p] = {}
 
 
 def _ctx(device: int) -> ctypes.c_void_p:
+    """The calling thread's ctx for ``device`` (a ctx is not thread-safe:
+    one per device per host thread, include/bpbc_sw.h)."""
+    key = (device, threading.get_ident())
     with _ctx_lock:
-        c = _ctxs.get(device)
+        c = _ctxs.get(key)
         if c is None:
             c = ctypes.c_void_p()
             check(_lib.load().bpbc_sw_init(device, ctypes.byref(c)))
-            _ctxs[device] = c
+            _ctxs[key] = c
         return c
 
 

@@ -244,3 +244,12 @@ def test_untranspose_kernel(lanes, s):
         red[:, b] = (((mx >> b) & 1).astype(np.uint64) << np.arange(32, dtype=np.uint64)
                      ).sum(axis=1).astype(np.uint32)
     np.testing.assert_array_equal(np.minimum(oracle.untranspose(red), cap)[:P], want)
+
+
+def test_multi_device_driver():
+    """score_multi_device shards over host threads (here twice cuda:0, one ctx
+    per thread) and reassembles; ragged P so shards differ in size."""
+    from paper_conf_ipps_nishimurabin17_b200 import parallel
+    q, t = synth.gen_pairs(2024, 3001, 64, 80, planted=True)
+    got = parallel.score_multi_device(q, t, 2, -1, -1, 8, devices=[0, 0, 0])
+    np.testing.assert_array_equal(got, oracle.sw_batch(q, t, 2, -1, -1, score_bits=8))
