@@ -21,7 +21,11 @@ struct bpbc_sw_ctx {
   uint8_t* d_t = nullptr;
   int32_t* d_out = nullptr;
   size_t d_q_bytes = 0, d_t_bytes = 0, d_out_bytes = 0;
-  cudaStream_t host_stream = nullptr;
+  // host path: two streams, chunk c of the batch runs on stream c % 2 with
+  // its own workspace, so chunk c+1's H2D overlaps chunk c's kernels
+  cudaStream_t host_streams[2] = {nullptr, nullptr};
+  void* ws_h[2] = {nullptr, nullptr};
+  size_t ws_h_bytes[2] = {0, 0};
   char err[512] = {0};
   // last plan
   int32_t plan_circuit = -1, plan_width = 0, plan_R = 0, plan_L = 0, plan_ops = 0;
@@ -186,10 +190,8 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   if (ctx->profiling)
     for (int i = 0; i < 4; ++i) ev[i] = ctx->take_event();
   if (ev[0]) cudaEventRecord(ev[0], st);
-  cudaError_t e = launch_pack(qx, P, mq, Xp, ctx->d_flags, ctx->num_sms, st);
-  if (e != cudaSuccess) return cuda_fail(ctx, e, "pack(query)");
-  e = launch_pack(ty, P, nt, Yp, ctx->d_flags, ctx->num_sms, st);
-  if (e != cudaSuccess) return cuda_fail(ctx, e, "pack(target)");
+  cudaError_t e = launch_pack2(qx, mq, Xp, ty, nt, Yp, P, ctx->d_flags, ctx->num_sms, st);
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "pack");
 
   if (ev[1]) cudaEventRecord(ev[1], st);
   std::call_once(g_table_once, init_table);
@@ -335,7 +337,10 @@ int bpbc_sw_destroy(bpbc_sw_ctx* ctx) {
   if (ctx->d_q) cudaFree(ctx->d_q);
   if (ctx->d_t) cudaFree(ctx->d_t);
   if (ctx->d_out) cudaFree(ctx->d_out);
-  if (ctx->host_stream) cudaStreamDestroy(ctx->host_stream);
+  for (int i = 0; i < 2; ++i) {
+    if (ctx->host_streams[i]) cudaStreamDestroy(ctx->host_streams[i]);
+    if (ctx->ws_h[i]) cudaFree(ctx->ws_h[i]);
+  }
   for (cudaEvent_t e : ctx->ev_pool) cudaEventDestroy(e);
   delete ctx;
   return BPBC_OK;
@@ -385,29 +390,50 @@ int bpbc_sw_score_batch_host(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8
   if (!query || !target || !out_scores) return BPBC_ERR_INVALID_ARG;
   DeviceGuard dg(ctx->device);
   cudaError_t e;
-  if (!ctx->host_stream) {
-    e = cudaStreamCreateWithFlags(&ctx->host_stream, cudaStreamNonBlocking);
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaStreamCreate");
+  for (int i = 0; i < 2; ++i) {
+    if (!ctx->host_streams[i]) {
+      e = cudaStreamCreateWithFlags(&ctx->host_streams[i], cudaStreamNonBlocking);
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaStreamCreate");
+    }
   }
   const size_t qb = size_t(num_pairs) * m, tb = size_t(num_pairs) * n,
                ob = size_t(num_pairs) * sizeof(int32_t);
+  // chunks of >= 64K pairs (multiples of 32), at most 8
+  int64_t nchunks = (num_pairs + 65535) / 65536;
+  if (nchunks > 8) nchunks = 8;
+  if (nchunks < 1) nchunks = 1;
+  int64_t chunk = (num_pairs + nchunks - 1) / nchunks;
+  chunk = (chunk + 31) / 32 * 32;
   size_t need = 0;
-  bpbc_sw_workspace_bytes(num_pairs, m, n, &need);
+  bpbc_sw_workspace_bytes(chunk < num_pairs ? chunk : num_pairs, m, n, &need);
   if ((rc = grow(ctx, (void**)&ctx->d_q, &ctx->d_q_bytes, qb, "cudaMalloc(q)")) != BPBC_OK) return rc;
   if ((rc = grow(ctx, (void**)&ctx->d_t, &ctx->d_t_bytes, tb, "cudaMalloc(t)")) != BPBC_OK) return rc;
   if ((rc = grow(ctx, (void**)&ctx->d_out, &ctx->d_out_bytes, ob, "cudaMalloc(out)")) != BPBC_OK)
     return rc;
-  if ((rc = ensure_ws(ctx, need)) != BPBC_OK) return rc;
-  cudaStream_t st = ctx->host_stream;
-  e = cudaMemcpyAsync(ctx->d_q, query, qb, cudaMemcpyHostToDevice, st);
-  if (e == cudaSuccess) e = cudaMemcpyAsync(ctx->d_t, target, tb, cudaMemcpyHostToDevice, st);
-  if (e != cudaSuccess) return cuda_fail(ctx, e, "H2D");
-  rc = run_device(ctx, ctx->d_q, ctx->d_t, num_pairs, m, n, match, mismatch, gap, score_bits,
-                  ctx->d_out, static_cast<uint8_t*>(ctx->ws), st);
-  if (rc != BPBC_OK) return rc;
-  e = cudaMemcpyAsync(out_scores, ctx->d_out, ob, cudaMemcpyDeviceToHost, st);
-  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-  if (e != cudaSuccess) return cuda_fail(ctx, e, "D2H");
+  for (int i = 0; i < 2; ++i)
+    if ((rc = grow(ctx, &ctx->ws_h[i], &ctx->ws_h_bytes[i], need, "cudaMalloc(workspace)")) !=
+        BPBC_OK)
+      return rc;
+  for (int64_t c0 = 0, ci = 0; c0 < num_pairs; c0 += chunk, ++ci) {
+    const int64_t cp = num_pairs - c0 < chunk ? num_pairs - c0 : chunk;
+    cudaStream_t st = ctx->host_streams[ci & 1];
+    e = cudaMemcpyAsync(ctx->d_q + c0 * m, query + c0 * m, size_t(cp) * m,
+                        cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(ctx->d_t + c0 * n, target + c0 * n, size_t(cp) * n,
+                          cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "H2D");
+    rc = run_device(ctx, ctx->d_q + c0 * m, ctx->d_t + c0 * n, cp, m, n, match, mismatch, gap,
+                    score_bits, ctx->d_out + c0, static_cast<uint8_t*>(ctx->ws_h[ci & 1]), st);
+    if (rc != BPBC_OK) return rc;
+    e = cudaMemcpyAsync(out_scores + c0, ctx->d_out + c0, size_t(cp) * sizeof(int32_t),
+                        cudaMemcpyDeviceToHost, st);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "D2H");
+  }
+  for (int i = 0; i < 2; ++i) {
+    e = cudaStreamSynchronize(ctx->host_streams[i]);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "sync");
+  }
   return BPBC_OK;
 }
 

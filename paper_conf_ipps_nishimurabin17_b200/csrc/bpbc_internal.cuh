@@ -66,7 +66,11 @@ BPBC_DECLARE_REG(15)
 BPBC_DECLARE_REG(16)
 #undef BPBC_DECLARE_REG
 
-// pack.cu
+// pack.cu: one launch packs up to two [num_pairs][len] code arrays (query and
+// target); a job with codes == nullptr is skipped.
+cudaError_t launch_pack2(const uint8_t* codes_a, int len_a, uint2* planes_a,
+                         const uint8_t* codes_b, int len_b, uint2* planes_b, int64_t num_pairs,
+                         uint32_t* flags, int num_sms, cudaStream_t stream);
 cudaError_t launch_pack(const uint8_t* codes, int64_t num_pairs, int len, uint2* planes,
                         uint32_t* flags, int num_sms, cudaStream_t stream);
 // extract.cu

@@ -195,10 +195,14 @@ BPBC_HD void ssub_run(const uint32_t (&X)[S], const uint32_t* gm, uint32_t (&U)[
 // kill forces H = 0 (rows past m).  LOP3 per word-cell:
 //   2 + (2S - 1) + 4S + (2S - 1) = 8S, 10S with the running max
 //   (S = 9: 90; the paper's Theorem 6 + Lemma 2 count 57S - 19 = 494).
+//
+// Dp receives D' (the diagonal term).  The running maximum is taken over D'
+// instead of H (see finish_exact below), so it never waits for the
+// comparator chain.
 template <int S, class K, bool KILL>
 BPBC_HD void cell_exact(const uint32_t (&up)[S], const uint32_t (&left)[S],
                         const uint32_t (&diag)[S], uint32_t xh, uint32_t xl, uint32_t yh,
-                        uint32_t yl, uint32_t kill, uint32_t (&H)[S]) {
+                        uint32_t yl, uint32_t kill, uint32_t (&H)[S], uint32_t (&Dp)[S]) {
   static_assert(K::kFixed && K::g >= K::c2, "exact cell needs compile-time g >= c2");
   constexpr int A = K::c1 + K::g, B = K::g - K::c2;
   const uint32_t e = mismatch_flag(xh, xl, yh, yl);
@@ -214,6 +218,21 @@ BPBC_HD void cell_exact(const uint32_t (&up)[S], const uint32_t (&left)[S],
   mux<S>(lt<S>(up, left), up, left, T);
   mux<S>(lt<S>(T, D), T, D, X);
   ssub_const<S, K::g, KILL>(X, kill, H);
+#pragma unroll
+  for (int i = 0; i < S; ++i) Dp[i] = D[i];
+}
+
+// Maximum over cells taken on the diagonal term.  The cell holding the
+// largest score H* > 0 got it from its diagonal input: if H* came from
+// up - g or left - g, that neighbour would hold H* + g > H*.  Every D <= H.
+// Hence max_ij H = max(0, max_ij D) with D = diag + w (saturating cell), and
+// max_ij H = max(0, max_ij D' - g) with D' = diag + w + g (exact cell).  The
+// lane keeps M over D (2S LOP3 per cell, as over H) and the exact kernel
+// subtracts g once per group (finish_exact).  D is ready long before H, so
+// the M chain runs beside the comparator chain instead of after it.
+template <int S, int G>
+BPBC_HD void finish_exact(const uint32_t (&Mp)[S], uint32_t (&M)[S]) {
+  ssub_const<S, G, false>(Mp, 0u, M);
 }
 
 // ---------------------------------------------------------------------------
@@ -226,10 +245,11 @@ BPBC_HD void cell_exact(const uint32_t (&up)[S], const uint32_t (&left)[S],
 //   H = max(D, U)
 // LOP3 per word-cell with compile-time constants: 2 + 2S + 2S + 3S + 2S =
 // 9S + 2, 11S + 2 with the running max.
+// D receives the diagonal term (see finish_exact above).
 template <int S, class K>
 BPBC_HD void cell_sat(const uint32_t (&up)[S], const uint32_t (&left)[S],
                       const uint32_t (&diag)[S], uint32_t xh, uint32_t xl, uint32_t yh,
-                      uint32_t yl, uint32_t (&H)[S], const K& k) {
+                      uint32_t yl, uint32_t (&H)[S], uint32_t (&D)[S], const K& k) {
   const uint32_t e = mismatch_flag(xh, xl, yh, yl);
   uint32_t T[S], U[S];
   mux<S>(lt<S>(up, left), up, left, T);
@@ -238,7 +258,7 @@ BPBC_HD void cell_sat(const uint32_t (&up)[S], const uint32_t (&left)[S],
   } else {
     ssub_run<S>(T, k.gmask, U);
   }
-  uint32_t s[S], D[S];
+  uint32_t s[S];
   uint32_t c = 0u;
   if constexpr (K::kFixed) {
     constexpr int N = ((1 << S) - K::c2) & ((1 << S) - 1);  // mismatch operand

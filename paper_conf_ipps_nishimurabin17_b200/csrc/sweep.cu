@@ -93,6 +93,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     }
   }
   const uint2* yp = a.Yp + gb * a.n - sl;
+  uint2 ynext = __ldg(yp);
   int cnt = sl;      // steps until my next group starts (J % n == 0)
   int64_t gi = -1;   // my current group within the stream
 
@@ -104,8 +105,15 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     if (cnt == 0) {  // column 0 of my next group (divergent, once per group)
       if (gi >= 0 && gi < Gs) {
         uint32_t* dst = a.Mpart + ((gb + gi) * L + sl) * S;
+        if constexpr (CIRC == kExact) {
+          uint32_t F[S];
+          finish_exact<S, K::g>(M, F);  // M tracked D' = diag + w + g
 #pragma unroll
-        for (int i = 0; i < S; ++i) dst[i] = M[i];
+          for (int i = 0; i < S; ++i) dst[i] = F[i];
+        } else {
+#pragma unroll
+          for (int i = 0; i < S; ++i) dst[i] = M[i];
+        }
       }
       ++gi;
 #pragma unroll
@@ -130,7 +138,8 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     }
     --cnt;
 
-    const uint2 y = __ldg(yp + tau);
+    const uint2 y = ynext;
+    ynext = __ldg(yp + tau + 1);  // prefetch one step ahead (pads cover it)
     uint32_t dg[S], u[S];
 #pragma unroll
     for (int i = 0; i < S; ++i) {
@@ -139,14 +148,15 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     }
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-      uint32_t hn[S];
+      uint32_t hn[S], dn[S];
+      // running max over the diagonal term (circuit.cuh finish_exact); padded
+      // rows are masked out of it
       if constexpr (CIRC == kExact) {
-        cell_exact<S, K, PAD>(u, H[r], dg, xh[r], xl[r], y.x, y.y, kill[r], hn);
-        runmax<S, false>(M, hn, 0u);
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn);
       } else {
-        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, k);
-        runmax<S, PAD>(M, hn, kill[r]);
+        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
       }
+      runmax<S, PAD>(M, dn, kill[r]);
 #pragma unroll
       for (int i = 0; i < S; ++i) {
         dg[i] = H[r][i];

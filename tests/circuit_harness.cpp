@@ -43,15 +43,15 @@ void unslice(const uint32_t (&w)[S], int* v) {
 template <int S>
 void cell(int circuit, const KRun& kr, const uint32_t (&up)[S], const uint32_t (&left)[S],
           const uint32_t (&diag)[S], uint32_t xh, uint32_t xl, uint32_t yh, uint32_t yl,
-          uint32_t kill, uint32_t (&H)[S]) {
+          uint32_t kill, uint32_t (&H)[S], uint32_t (&D)[S]) {
   using K = KFix<2, 1, 1>;
   if (circuit == 0) {
-    if (kill) cell_exact<S, K, true>(up, left, diag, xh, xl, yh, yl, kill, H);
-    else cell_exact<S, K, false>(up, left, diag, xh, xl, yh, yl, 0u, H);
+    if (kill) cell_exact<S, K, true>(up, left, diag, xh, xl, yh, yl, kill, H, D);
+    else cell_exact<S, K, false>(up, left, diag, xh, xl, yh, yl, 0u, H, D);
   } else if (circuit == 1) {
-    cell_sat<S, K>(up, left, diag, xh, xl, yh, yl, H, K{});
+    cell_sat<S, K>(up, left, diag, xh, xl, yh, yl, H, D, K{});
   } else {
-    cell_sat<S, KRun>(up, left, diag, xh, xl, yh, yl, H, kr);
+    cell_sat<S, KRun>(up, left, diag, xh, xl, yh, yl, H, D, kr);
   }
 }
 
@@ -62,21 +62,23 @@ long long exhaustive(int circuit, int c1, int c2, int g, int with_kill) {
   const KRun kr = make_krun(S, c1, c2, g);
   const int cap = (1 << S) - 1;
   long long bad = 0;
-  int up[32], left[32], diag[32], ref[32], got[32];
+  int up[32], left[32], diag[32], ref[32], got[32], refd[32], gotd[32];
   uint32_t eword = 0;
   int cnt = 0;
   auto flush = [&](int n) {
-    uint32_t U[S], Lf[S], D[S], H[S];
+    uint32_t U[S], Lf[S], D[S], H[S], Dt[S];
     slice<S>(up, U);
     slice<S>(left, Lf);
     slice<S>(diag, D);
     // x = A (code 0) everywhere; y = A where e = 0, T (code 1) where e = 1
     const uint32_t kill = with_kill ? 0xAAAAAAAAu : 0u;
-    cell<S>(circuit, kr, U, Lf, D, 0u, 0u, 0u, eword, kill, H);
+    cell<S>(circuit, kr, U, Lf, D, 0u, 0u, 0u, eword, kill, H, Dt);
     unslice<S>(H, got);
+    unslice<S>(Dt, gotd);
     for (int k = 0; k < n; ++k) {
       const int expect = (kill >> k) & 1 ? 0 : ref[k];
       if (got[k] != expect) ++bad;
+      if (gotd[k] != refd[k]) ++bad;  // diagonal term (running-max input)
     }
   };
   for (int a = 0; a <= cap; ++a)
@@ -88,11 +90,13 @@ long long exhaustive(int circuit, int c1, int c2, int g, int with_kill) {
             // exact circuit domain: no intermediate above the cap
             if (d + c1 + g > cap || a > cap - 0 || b > cap) continue;
             r = imax(0, imax(a - g, imax(b - g, d + (e ? -c2 : c1))));
+            refd[cnt] = d + (e ? -c2 : c1) + g;  // D' = diag + w + g
           } else {
             const int T = imax(a, b);
             const int U = imax(T - g, 0);
             const int D = e ? imax(d - c2, 0) : (d + c1 > cap ? cap : d + c1);
             r = imax(U, D);
+            refd[cnt] = D;
           }
           up[cnt] = a;
           left[cnt] = b;
@@ -123,21 +127,27 @@ void group_dp(int circuit, int c1, int c2, int g, const uint32_t* xp, int m, con
   for (int r = 0; r < m; ++r) {
     for (int i = 0; i < S; ++i) cur[0][i] = 0;
     for (int j = 1; j <= n; ++j) {
-      uint32_t up[S], left[S], diag[S], H[S];
+      uint32_t up[S], left[S], diag[S], H[S], D[S];
       for (int i = 0; i < S; ++i) {
         up[i] = prev[j][i];
         left[i] = cur[j - 1][i];
         diag[i] = prev[j - 1][i];
       }
       cell<S>(circuit, kr, up, left, diag, xp[2 * r], xp[2 * r + 1], yp[2 * (j - 1)],
-              yp[2 * (j - 1) + 1], 0u, H);
-      runmax<S, false>(M, H, 0u);
+              yp[2 * (j - 1) + 1], 0u, H, D);
+      runmax<S, false>(M, D, 0u);  // max over the diagonal term (finish_exact)
       for (int i = 0; i < S; ++i) cur[j][i] = H[i];
     }
     for (int j = 0; j <= n; ++j)
       for (int i = 0; i < S; ++i) prev[j][i] = cur[j][i];
   }
-  for (int i = 0; i < S; ++i) Mout[i] = M[i];
+  if (circuit == 0) {
+    uint32_t F[S];
+    finish_exact<S, 1>(M, F);  // KFix<2,1,1>: g = 1
+    for (int i = 0; i < S; ++i) Mout[i] = F[i];
+  } else {
+    for (int i = 0; i < S; ++i) Mout[i] = M[i];
+  }
 }
 
 }  // namespace

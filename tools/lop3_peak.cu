@@ -1,0 +1,86 @@
+// lop3_peak.cu -- micro-benchmark of the B200 integer-logic (alu pipe) peak:
+// the roofline denominator of the sweep kernel.
+//
+// Every thread runs 8 independent chains of lop3.b32 (the same gate kind the
+// sweep issues), full occupancy, grid = 148 SMs x 8 blocks of 256 threads.
+// Prints lane-ops/s, lane-ops per SM-clock (from the measured SM clock via
+// clock64 on one SM) and the implied lanes/clk/SM.
+//
+// build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o lop3_peak lop3_peak.cu
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+template <int LUT>
+__device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm volatile("lop3.b32 %0, %1, %2, %3, %4;" : "=r"(d) : "r"(a), "r"(b), "r"(c), "n"(LUT));
+  return d;
+}
+
+__global__ void __launch_bounds__(256) peak_kernel(uint32_t* out, int iters, long long* cyc) {
+  uint32_t a[8], b = threadIdx.x * 0x9E3779B9u, c = blockIdx.x * 0x85EBCA6Bu;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) a[k] = b ^ (k * 0x27D4EB2Fu);
+  long long t0 = clock64();
+  for (int i = 0; i < iters; ++i) {
+#pragma unroll
+    for (int u = 0; u < 16; ++u) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) a[k] = lop3<0xE8>(a[k], b, c);  // MAJ: the carry gate
+    }
+  }
+  long long t1 = clock64();
+  uint32_t r = 0;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) r ^= a[k];
+  if (r == 0x12345678u) out[0] = r;  // keep the chains alive
+  if (threadIdx.x == 0 && blockIdx.x == 0) *cyc = t1 - t0;
+}
+
+int main() {
+  int dev = 0, sms = 0, clk_khz = 0;
+  cudaSetDevice(dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaDeviceGetAttribute(&clk_khz, cudaDevAttrClockRate, dev);
+  uint32_t* out;
+  long long* cyc;
+  cudaMalloc(&out, 4);
+  cudaMalloc(&cyc, 8);
+  const int block = 256, grid = sms * 8, iters = 4096;
+  peak_kernel<<<grid, block>>>(out, 64, cyc);  // warm-up
+  cudaDeviceSynchronize();
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  double best = 0, best_cyc_rate = 0;
+  for (int rep = 0; rep < 5; ++rep) {
+    cudaEventRecord(e0);
+    peak_kernel<<<grid, block>>>(out, iters, cyc);
+    cudaEventRecord(e1);
+    cudaEventSynchronize(e1);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    long long c = 0;
+    cudaMemcpy(&c, cyc, 8, cudaMemcpyDeviceToHost);
+    const double ops = double(grid) * block * iters * 16 * 8;
+    const double rate = ops / (ms * 1e-3);
+    // per-SM clock implied by the first block's cycle count over the kernel
+    const double mhz = double(c) / (ms * 1e-3) / 1e6;
+    if (rate > best) {
+      best = rate;
+      best_cyc_rate = mhz;
+    }
+  }
+  // lanes per SM-clock: ops / (SMs * cycles); cycles = time * clock
+  const double lanes = best / (sms * best_cyc_rate * 1e6);
+  printf("{\"lop3_lane_ops_per_s\": %.4e, \"sm_clock_mhz_from_clock64\": %.1f, "
+         "\"lanes_per_clk_per_sm\": %.2f, \"sms\": %d, \"attr_clock_mhz\": %.1f}\n",
+         best, best_cyc_rate, lanes, sms, clk_khz / 1e3);
+  cudaError_t err = cudaGetLastError();
+  if (err != cudaSuccess) {
+    printf("error: %s\n", cudaGetErrorString(err));
+    return 1;
+  }
+  return 0;
+}
