@@ -40,11 +40,13 @@ if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
 
 METRIC = "GCUPS (bit-exact max local score)"
-CONFIGS = {
-    1: dict(P=1024, m=64, n=64, s=8),
-    2: dict(P=1 << 20, m=128, n=128, s=9),
-    3: dict(P=1 << 22, m=256, n=256, s=10),
-    4: dict(P=1 << 20, m=64, n=1024, s=8),
+CONFIGS = {  # BASELINE.json configs; "scaling" says how N GPUs split it
+    1: dict(P=1024, m=64, n=64, s=8, scaling="weak"),
+    2: dict(P=1 << 20, m=128, n=128, s=9, scaling="weak"),
+    3: dict(P=1 << 22, m=256, n=256, s=10, scaling="strong"),  # 2^22 pairs sharded over N
+    4: dict(P=1 << 20, m=64, n=1024, s=8, scaling="weak"),
+    5: dict(P=1 << 22, m=512, n=512, s=11, scaling="weak"),  # one point of the C5 sweep
+    6: dict(P=32768, m=128, n=65536, s=9, scaling="weak"),  # the paper's own shape
 }
 CONSTS = (2, -1, -1)  # match, mismatch, gap (Table II, reading R14)
 SM_COUNT = 148
@@ -52,7 +54,8 @@ ALU_LANES_PER_SM_CLK = 64  # 4 SMSP x 16 lanes/clk (LOP3 rt = 2 cyc per warp ins
 
 
 def workload_name(cid, c):
-    return (f"C{cid}: {c['P']} DNA pairs, m={c['m']}, n={c['n']}, "
+    name = "paper shape (P:L382)" if cid == 6 else f"C{cid}"
+    return (f"{name}: {c['P']} DNA pairs, m={c['m']}, n={c['n']}, "
             f"match/mismatch/gap = +2/-1/-1, {c['s']}-bit score slices, max score only")
 
 
@@ -172,7 +175,8 @@ def run_reference(args, cfg):
     line = {"metric": METRIC, "value": round(v, 4), "unit": "GCUPS", "impl": "reference",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "scaling": cfg["scaling"], "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic",
             "config": {"workload": workload_name(cfg["id"], cfg),
                        "sample_pairs_per_step": per_step},
             "cpu_baseline": {"value": round(v, 4), "unit": "GCUPS", "cores": threads,
@@ -193,6 +197,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--score-bits", type=int, default=None)
+    ap.add_argument("--m", type=int, default=None, help="override the query length")
+    ap.add_argument("--n", type=int, default=None, help="override the target length")
+    ap.add_argument("--pairs", type=int, default=None, help="override the pair count")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
@@ -200,6 +207,9 @@ def main():
     cfg["id"] = args.config
     if args.score_bits:
         cfg["s"] = args.score_bits
+    for key, val in (("m", args.m), ("n", args.n), ("P", args.pairs)):
+        if val:
+            cfg[key] = val
     if args.impl == "reference":
         run_reference(args, cfg)
         return
@@ -218,13 +228,21 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
-    P, m, n, s = cfg["P"], cfg["m"], cfg["n"], cfg["s"]
+    m, n, s = cfg["m"], cfg["n"], cfg["s"]
     seed = synth.seed_for_config(args.config)
+    from paper_conf_ipps_nishimurabin17_b200 import parallel
+    if cfg["scaling"] == "strong":  # the config's pairs split over the ranks
+        P_total = cfg["P"]
+        p0, p1 = parallel.shard_range(P_total, world, rank)
+    else:  # every rank scores a config-sized batch of its own
+        P_total = world * cfg["P"]
+        p0, p1 = rank * cfg["P"], (rank + 1) * cfg["P"]
+    P = p1 - p0
 
     # inputs: this rank's shard, generated on the host into pinned buffers
     hq = torch.empty((P, m), dtype=torch.uint8, pin_memory=True)
     ht = torch.empty((P, n), dtype=torch.uint8, pin_memory=True)
-    synth.gen_pairs(seed, P, m, n, p_offset=rank * P, out_q=hq.numpy(), out_t=ht.numpy())
+    synth.gen_pairs(seed, P, m, n, p_offset=p0, out_q=hq.numpy(), out_t=ht.numpy())
     dq = hq.to(dev, non_blocking=True)
     dt = ht.to(dev, non_blocking=True)
     out = torch.empty(P, dtype=torch.int32, device=dev)
@@ -266,7 +284,7 @@ def main():
         tt = torch.tensor([t_ms], dtype=torch.float64, device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t_ms = tt.item()
-    cells = world * P * m * n * args.steps
+    cells = P_total * m * n * args.steps
     gcups = cells / (t_ms / 1e3) / 1e9
 
     # ---------------- end to end through the host-buffer C call
@@ -287,15 +305,14 @@ def main():
             te = torch.tensor([el], dtype=torch.float64, device=dev)
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
             el = te.item()
-        e2e = {"value": round(world * P * m * n * ksteps / el / 1e9, 2), "unit": "GCUPS",
-               "h2d_bytes_per_step": world * P * (m + n), "d2h_bytes_per_step": world * P * 4,
+        e2e = {"value": round(P_total * m * n * ksteps / el / 1e9, 2), "unit": "GCUPS",
+               "h2d_bytes_per_step": P_total * (m + n), "d2h_bytes_per_step": P_total * 4,
                "steps": ksteps, "timing": "host wall clock around the blocking C call "
                                           "(pinned host buffers)"}
 
     # ---------------- result gather (outside the timed region) + parity sample
-    if world > 1:
-        from paper_conf_ipps_nishimurabin17_b200 import parallel
-        full = parallel.gather_scores(out, world * P)  # rank r holds pairs [rP, (r+1)P)
+    if world > 1:  # rank r holds the pairs of shard_range(P_total, world, r)
+        full = parallel.gather_scores(out, P_total)
         got_all = full.cpu().numpy()
     else:
         got_all = out.cpu().numpy()
@@ -304,8 +321,9 @@ def main():
         return
     import oracle
     rng = np.random.default_rng(seed)
-    total = world * P
-    idx = np.unique(np.concatenate([rng.choice(total, size=min(total, 2048), replace=False),
+    total = P_total
+    nsamp = int(min(total, 2048, max(16, 2e9 // (m * n))))  # ~2e9 oracle cells at most
+    idx = np.unique(np.concatenate([rng.choice(total, size=nsamp, replace=False),
                                     [0, total - 1]]))
     sq = np.empty((idx.size, m), dtype=np.uint8)
     st_ = np.empty((idx.size, n), dtype=np.uint8)
@@ -351,14 +369,16 @@ def main():
     line = {"metric": METRIC, "value": round(gcups, 2), "unit": "GCUPS", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(t_ms / args.steps, 4), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u32 bit-sliced (s-bit scores)",
+            "scaling": cfg["scaling"], "vs_baseline": None,
+            "dtype": "u32 bit-sliced (s-bit scores)",
             "data": "synthetic (seeded i.i.d. uniform DNA, SplitMix64)",
-            "config": {"workload": workload_name(args.config, cfg), "pairs_per_gpu": P,
+            "config": {"workload": workload_name(args.config, cfg), "pairs_per_gpu": P, "pairs_total": P_total,
                        "m": m, "n": n, "score_bits": s, "parallelism": f"dp{world} (pair shards)",
                        "l2": "inputs 320 MiB > 126 MB L2, plus a 256 MiB L2 flush between steps",
                        "plan": plan},
             "e2e": e2e, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,
-            "gpu_launches": 4 * args.steps * world, "parity": parity}
+            # ours per step and rank: pack (query+target), sweep, extract
+            "gpu_launches": 3 * args.steps * world, "parity": parity}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

@@ -64,7 +64,8 @@ typedef enum {
 /* Supported ranges of this build. */
 #define BPBC_MIN_SCORE_BITS 4
 #define BPBC_MAX_SCORE_BITS 16
-#define BPBC_MAX_LEN (1 << 20) /* m, n <= 2^20 */
+#define BPBC_MAX_LEN (1 << 20)       /* m, n <= 2^20 */
+#define BPBC_MAX_QUERY_LEN (1 << 16) /* min(m, n) <= 2^16 */
 
 /* Binds the context to `cuda_device`, creates its device flag word and
  * queries the SM count.  No pair-sized allocation.  *out_ctx is set only on
@@ -76,9 +77,11 @@ int bpbc_sw_init(int cuda_device, bpbc_sw_ctx **out_ctx);
 int bpbc_sw_destroy(bpbc_sw_ctx *ctx);
 
 /* Bytes of device workspace bpbc_sw_score_batch needs for these sizes:
- * the bit-transposed planes 8 * ceil(P/32) * (m + n) bytes plus padding and
- * the per-lane partial maxima (at most 2 KiB per 32-pair group per 256 query
- * rows).  Pure host function. */
+ * the bit-transposed planes 8 * ceil(P/32) * (m + n) bytes plus padding,
+ * the per-lane partial maxima (2 KiB per 32-pair group, per 128 query rows
+ * when min(m, n) > 256) and, when min(m, n) > 256, the stripe boundary rows
+ * (64 * max(m, n) bytes per concurrent group stream, at most 1 GiB).  Pure
+ * host function. */
 int bpbc_sw_workspace_bytes(int64_t num_pairs, int32_t m, int32_t n, size_t *bytes);
 
 /*
@@ -90,8 +93,9 @@ int bpbc_sw_workspace_bytes(int64_t num_pairs, int32_t m, int32_t n, size_t *byt
  * target      device, uint8 [num_pairs][n] row-major base codes (Y_k).
  * num_pairs   >= 0; 0 is a no-op.  Need not be a multiple of 32.
  * m, n        1 .. BPBC_MAX_LEN each; m > n is allowed (roles are swapped
- *             internally; the score is symmetric, R17).  min(m, n) <= 256
- *             in this build (else BPBC_ERR_UNSUPPORTED).
+ *             internally; the score is symmetric, R17).  min(m, n) <=
+ *             BPBC_MAX_QUERY_LEN (else BPBC_ERR_UNSUPPORTED); above 256 the
+ *             query rows are processed in stripes of 128.
  * match       >= 1                      (paper c1)
  * mismatch    <= 0                      (paper -c2)
  * gap         <= 0                      (paper -gap, linear per column)

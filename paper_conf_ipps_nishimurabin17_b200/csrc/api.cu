@@ -52,10 +52,25 @@ namespace bpbc {
 namespace {
 
 SweepEntry g_table[kNumVariants][kNumRL][13];
+SweepEntry g_striped[3][13];
 std::once_flag g_table_once;
 
 void init_table() {
   memset(g_table, 0, sizeof(g_table));
+  memset(g_striped, 0, sizeof(g_striped));
+  register_striped_s4(g_striped);
+  register_striped_s5(g_striped);
+  register_striped_s6(g_striped);
+  register_striped_s7(g_striped);
+  register_striped_s8(g_striped);
+  register_striped_s9(g_striped);
+  register_striped_s10(g_striped);
+  register_striped_s11(g_striped);
+  register_striped_s12(g_striped);
+  register_striped_s13(g_striped);
+  register_striped_s14(g_striped);
+  register_striped_s15(g_striped);
+  register_striped_s16(g_striped);
   register_sweep_s4(g_table);
   register_sweep_s5(g_table);
   register_sweep_s6(g_table);
@@ -89,7 +104,9 @@ int cuda_fail(bpbc_sw_ctx* ctx, cudaError_t e, const char* what) {
 // offsets 256-byte aligned.
 struct Layout {
   int64_t G = 0;
-  int64_t x_off = 0, y_off = 0, mp_off = 0, total = 0;
+  int stripes = 1;             // > 1 only for the long-query (striped) kernel
+  int64_t bnd_streams = 0;     // streams the boundary buffer has room for
+  int64_t x_off = 0, y_off = 0, mp_off = 0, bnd_off = 0, zero_off = 0, total = 0;
 };
 
 int64_t align256(int64_t v) { return (v + 255) & ~int64_t(255); }
@@ -97,14 +114,26 @@ int64_t align256(int64_t v) { return (v + 255) & ~int64_t(255); }
 Layout layout(int64_t P, int mq, int nt) {
   Layout L;
   L.G = (P + 31) / 32;
+  // room for the striped kernel whenever the plan may pick it (m > 128)
+  L.stripes = mq > kStripeRows ? (mq + kStripeRows - 1) / kStripeRows : 1;
   const int64_t xbytes = (L.G * mq + kXBackPad) * 8;
   const int64_t ybytes = (kYFrontPad + L.G * nt + nt + kYBackPadExtra) * 8;
-  const int64_t stripes = (mq + 255) / 256;
-  const int64_t mpbytes = L.G * stripes * 32 * 16 * 4;
+  const int64_t mpbytes = L.G * L.stripes * 32 * 16 * 4;
+  int64_t bnd_bytes = 0;
+  if (L.stripes > 1) {
+    const int64_t per_stream = int64_t(nt) * 16 * 4;  // [n][16 words] at most
+    int64_t st = L.G < kMaxStripeStreams ? L.G : kMaxStripeStreams;
+    if (st * per_stream > kMaxBoundaryBytes) st = kMaxBoundaryBytes / per_stream;
+    if (st < 1) st = 1;
+    L.bnd_streams = st;
+    bnd_bytes = st * per_stream;
+  }
   L.x_off = 0;
   L.y_off = align256(xbytes);
   L.mp_off = L.y_off + align256(ybytes);
-  L.total = L.mp_off + align256(mpbytes);
+  L.bnd_off = L.mp_off + align256(mpbytes);
+  L.zero_off = L.bnd_off + align256(bnd_bytes);
+  L.total = L.zero_off + 256;
   return L;
 }
 
@@ -119,9 +148,11 @@ int make_plan(int mq, int c1, int c2, int g, int S, Plan* p) {
   if (mq <= 32) p->rl = 0;
   else if (mq <= 64) p->rl = 1;
   else if (mq <= 128) p->rl = 2;
-  else if (mq <= 256) p->rl = 3;
+  else if (mq <= kMaxShortRows) p->rl = 3;
+  else if (mq <= BPBC_MAX_QUERY_LEN) p->rl = -1;  // striped long-query kernel
   else return BPBC_ERR_UNSUPPORTED;
-  p->pad = mq != kRLR[p->rl] * kRLL[p->rl];
+  p->pad = p->rl < 0 || mq != kRLR[p->rl] * kRLL[p->rl];
+  const bool wide_r8 = p->rl == 3;  // R = 8 rows per lane: register-heavy at large S
   p->cap = (1 << S) - 1;
   const bool spec = (c1 == 2 && c2 == 1 && g == 1);
   // width of the saturating circuit: no saturation can happen at or above
@@ -141,12 +172,20 @@ int make_plan(int mq, int c1, int c2, int g, int S, Plan* p) {
       p->consts = kC211;
       p->width = s_ex;
       p->ops = 10 * s_ex;
+      if (wide_r8 && s_ex >= 13) {
+        p->rl = -1;
+        p->pad = true;
+      }
       return BPBC_OK;
     }
   }
   p->circuit = kSat;
   p->consts = spec ? kC211 : kCRun;
   p->width = s_sat;
+  if (wide_r8 && s_sat >= 13) {  // R = 8 x 13+ planes spills: use 128-row stripes
+    p->rl = -1;
+    p->pad = true;
+  }
   p->ops = spec ? cost_sat : 13 * s_sat + 4;  // runtime masks: +S (w), +S (ssub), +2
   return BPBC_OK;
 }
@@ -158,7 +197,7 @@ int validate_common(int64_t P, int m, int n, int match, int mismatch, int gap, i
   const int64_t cap = (int64_t(1) << S) - 1;
   if (match > cap || -int64_t(mismatch) > cap || -int64_t(gap) > cap) return BPBC_ERR_INVALID_ARG;
   if (m > BPBC_MAX_LEN || n > BPBC_MAX_LEN) return BPBC_ERR_UNSUPPORTED;
-  if ((m < n ? m : n) > 256) return BPBC_ERR_UNSUPPORTED;
+  if ((m < n ? m : n) > BPBC_MAX_QUERY_LEN) return BPBC_ERR_UNSUPPORTED;
   return BPBC_OK;
 }
 
@@ -195,16 +234,21 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
 
   if (ev[1]) cudaEventRecord(ev[1], st);
   std::call_once(g_table_once, init_table);
+  const bool striped = plan.rl < 0;
   const SweepEntry ent =
-      g_table[variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl][plan.width - 4];
+      striped ? g_striped[plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]
+                         [plan.width - 4]
+              : g_table[variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl]
+                       [plan.width - 4];
   if (!ent.launch) return BPBC_ERR_UNSUPPORTED;
-  const int R = kRLR[plan.rl], L = kRLL[plan.rl];
+  const int R = striped ? kStripeR : kRLR[plan.rl], L = striped ? 32 : kRLL[plan.rl];
   int nb = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, ent.func, 128, 0);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "occupancy");
   if (nb < 1) nb = 1;
   const int64_t segs = 32 / L;
-  const int64_t cap_streams = int64_t(ctx->num_sms) * nb * 4 * segs;
+  int64_t cap_streams = int64_t(ctx->num_sms) * nb * 4 * segs;
+  if (striped && cap_streams > lay.bnd_streams) cap_streams = lay.bnd_streams;
   SweepArgs a;
   a.Xp = Xp;
   a.Yp = Yp;
@@ -215,7 +259,14 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   a.streams = lay.G < cap_streams ? lay.G : cap_streams;
   a.base = lay.G / a.streams;
   a.rem = lay.G % a.streams;
-  a.steps = (a.base + (a.rem > 0 ? 1 : 0)) * int64_t(nt) + L;
+  a.stripes = striped ? (mq + kStripeRows - 1) / kStripeRows : 1;
+  a.bnd = reinterpret_cast<uint32_t*>(ws + lay.bnd_off);
+  a.bzero = reinterpret_cast<const uint32_t*>(ws + lay.zero_off);
+  a.steps = (a.base + (a.rem > 0 ? 1 : 0)) * a.stripes * int64_t(nt) + L;
+  if (striped) {
+    e = cudaMemsetAsync(ws + lay.zero_off, 0, 256, st);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "memset(zero row)");
+  }
   const int64_t warps = (a.streams + segs - 1) / segs;
   const int grid = int((warps + 3) / 4);
   KRun kr;
@@ -231,7 +282,7 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(ctx, e, "sweep");
   if (ev[2]) cudaEventRecord(ev[2], st);
-  e = launch_extract(Mpart, lay.G, L, W, P, plan.cap, out, ctx->num_sms, st);
+  e = launch_extract(Mpart, lay.G, L * a.stripes, W, P, plan.cap, out, ctx->num_sms, st);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "extract");
   if (ev[3]) cudaEventRecord(ev[3], st);
 

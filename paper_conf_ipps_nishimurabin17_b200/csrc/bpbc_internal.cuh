@@ -33,8 +33,19 @@ struct SweepArgs {
   int64_t streams;   // number of group streams (one per L lanes)
   int64_t base;      // groups per stream: base or base+1
   int64_t rem;       //   (the first rem streams get base+1)
-  int64_t steps;     // wavefront steps = (base + (rem>0)) * n + L
+  int64_t steps;     // wavefront steps = (base + (rem>0)) * stripes * n + L
+  // long-query (striped) kernel only
+  int stripes;          // row stripes of kStripeRows per group (1 = short kernel)
+  uint32_t* bnd;        // [streams][n][SP] stripe boundary rows
+  const uint32_t* bzero;  // 16 zero words
 };
+
+// Long queries: stripes of kStripeR rows per lane x 32 lanes.
+constexpr int kStripeR = 4;
+constexpr int kStripeRows = 32 * kStripeR;
+constexpr int kMaxShortRows = 256;     // m <= 256: the short kernel
+constexpr int64_t kMaxStripeStreams = 4096;
+constexpr int64_t kMaxBoundaryBytes = int64_t(1) << 30;
 
 typedef void (*SweepLaunchFn)(const SweepArgs&, const KRun&, int grid, int block,
                               cudaStream_t stream);
@@ -65,6 +76,23 @@ BPBC_DECLARE_REG(14)
 BPBC_DECLARE_REG(15)
 BPBC_DECLARE_REG(16)
 #undef BPBC_DECLARE_REG
+// Striped kernels: [0] exact (+2,-1,-1), [1] saturating (+2,-1,-1),
+// [2] saturating runtime constants; index S - 4.
+#define BPBC_DECLARE_SREG(S) void register_striped_s##S(SweepEntry (*tab)[13]);
+BPBC_DECLARE_SREG(4)
+BPBC_DECLARE_SREG(5)
+BPBC_DECLARE_SREG(6)
+BPBC_DECLARE_SREG(7)
+BPBC_DECLARE_SREG(8)
+BPBC_DECLARE_SREG(9)
+BPBC_DECLARE_SREG(10)
+BPBC_DECLARE_SREG(11)
+BPBC_DECLARE_SREG(12)
+BPBC_DECLARE_SREG(13)
+BPBC_DECLARE_SREG(14)
+BPBC_DECLARE_SREG(15)
+BPBC_DECLARE_SREG(16)
+#undef BPBC_DECLARE_SREG
 
 // pack.cu: one launch packs up to two [num_pairs][len] code arrays (query and
 // target); a job with codes == nullptr is skipped.

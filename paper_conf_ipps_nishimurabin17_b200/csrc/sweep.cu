@@ -169,12 +169,208 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   }
 }
 
+__device__ __forceinline__ uint32_t mad_lo(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t r;
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
+  return r;
+}
+
+// ---------------------------------------------------------------------------
+// Long queries (m > 256 after the R17 swap): the query rows are cut into
+// stripes of kStripeRows = L*R = 128 rows.  Every (group, stripe) pair is a
+// "unit" of n columns; a stream walks units group-major (g0s0, g0s1, ...,
+// g1s0, ...) exactly as the short kernel walks groups.  The bottom row of
+// stripe k (S planes per column) is handed to the top lane of stripe k+1
+// through a per-stream boundary buffer in global memory: the last lane stores
+// it at column j, and lane 0 of the next unit loads it n - L steps later (so
+// n > L is required, which holds because n >= m > 256).  Lane 0 of stripe 0
+// reads a zero row instead (border d[-1][j] = 0).  The partial
+// maxima go to Mpart[g][k][lane] (the extract kernel reduces stripes x lanes).
+// Everything else is the short kernel (same circuits, same wavefront).
+template <int S, int CIRC, class K>
+__global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a, const K k) {
+  constexpr int R = kStripeR, L = 32, LR = L * R;
+  constexpr int SP = (S + 3) / 4 * 4;  // boundary words per column (uint4 aligned)
+  const int sl = threadIdx.x & 31;
+  const int64_t warp = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  if (warp >= a.streams) return;  // uniform per warp
+  const int64_t stream = warp;
+  const int64_t Gs = a.base + (stream < a.rem ? 1 : 0);
+  const int64_t gb = stream * a.base + (stream < a.rem ? stream : a.rem);
+  const int stripes = a.stripes;
+  const int64_t units = Gs * stripes;
+  const uint32_t nz = opaque(sl != 0 ? 1u : 0u);
+  uint32_t* bnd = a.bnd + stream * int64_t(a.n) * SP;  // [n][SP] of this stream
+  const uint32_t* zero = a.bzero;                      // SP zero words
+
+  uint32_t kill[R];
+  uint32_t H[R][S], dtop[S], M[S], bnext[S];
+#pragma unroll
+  for (int i = 0; i < S; ++i) {
+    dtop[i] = 0;
+    M[i] = 0;
+    bnext[i] = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) H[r][i] = 0;
+  }
+#pragma unroll
+  for (int r = 0; r < R; ++r) kill[r] = 0;
+  uint32_t xh[R], xl[R], nxh[R], nxl[R];
+  auto load_x = [&](int64_t u) {  // query planes of unit u (clamped)
+    u = u < units ? u : units - 1;
+    const int64_t g = gb + u / stripes;
+    const int kk = int(u % stripes);
+    const uint2* xp = a.Xp + g * a.m + kk * LR + sl * R;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const uint2 v = __ldg(xp + r);
+      nxh[r] = v.x;
+      nxl[r] = v.y;
+    }
+  };
+  load_x(0);
+#pragma unroll
+  for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
+  const uint2* ycol = a.Yp;  // my current target column (valid dummy before unit 0)
+  uint2 ynext = __ldg(ycol);
+  uint2 yfirst = __ldg(a.Yp + gb * a.n);  // column 0 of my next unit
+  const uint32_t* bcol = zero;  // boundary column I load next (lane 0 only)
+  int bstep = 0;                // words to advance bcol per step (SP or 0)
+  bool store_bnd = false;       // last lane, not the last stripe
+  int cnt = sl;
+  int64_t vi = -1;
+
+  for (int64_t tau = 0; tau < a.steps; ++tau) {
+    uint32_t up[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i)
+      up[i] = mad_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1), nz, bnext[i]);
+    uint2 y;
+    if (cnt == 0) {  // column 0 of my next unit (divergent, once per unit)
+      if (vi >= 0 && vi < units) {
+        const int64_t g = gb + vi / stripes;
+        const int kk = int(vi % stripes);
+        uint32_t* dst = a.Mpart + ((g * stripes + kk) * L + sl) * S;
+        if constexpr (CIRC == kExact) {
+          uint32_t F[S];
+          finish_exact<S, K::g>(M, F);
+#pragma unroll
+          for (int i = 0; i < S; ++i) dst[i] = F[i];
+        } else {
+#pragma unroll
+          for (int i = 0; i < S; ++i) dst[i] = M[i];
+        }
+      }
+      ++vi;
+      const int64_t uc = vi < units ? vi : units - 1;
+      const int64_t g = gb + uc / stripes;
+      const int kk = int(uc % stripes);
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        M[i] = 0;
+        dtop[i] = 0;
+#pragma unroll
+        for (int r = 0; r < R; ++r) H[r][i] = 0;
+      }
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        xh[r] = nxh[r];
+        xl[r] = nxl[r];
+        kill[r] = (kk * LR + sl * R + r >= a.m) ? 0xFFFFFFFFu : 0u;
+      }
+      load_x(vi + 1);
+      ycol = a.Yp + g * a.n;
+      y = yfirst;
+      {
+        const int64_t un = vi + 1 < units ? vi + 1 : units - 1;
+        yfirst = __ldg(a.Yp + (gb + un / stripes) * a.n);
+      }
+      const bool from_bnd = sl == 0 && kk > 0;
+      bcol = from_bnd ? bnd : zero;
+      bstep = from_bnd ? SP : 0;
+      store_bnd = sl == L - 1 && kk + 1 < stripes;
+      if (from_bnd) {  // column 0 of a lower stripe: up = boundary row 0
+#pragma unroll
+        for (int i = 0; i < S; ++i) up[i] = __ldcg(bnd + i);
+      }
+      cnt = a.n;
+    } else {
+      y = ynext;
+      ++ycol;
+    }
+    --cnt;
+    ynext = __ldg(ycol + 1);
+    // boundary row for the next step (lane 0 of stripes > 0; zeros otherwise;
+    // column 0 of a unit is loaded at the switch instead)
+    {
+      const uint32_t* bp = bcol + (cnt > 0 ? bstep : 0);
+      const uint4* b4 = reinterpret_cast<const uint4*>(cnt > 0 ? bp : zero);
+#pragma unroll
+      for (int q = 0; q < SP / 4; ++q) {
+        const uint4 v = __ldcg(b4 + q);
+        if (4 * q + 0 < S) bnext[4 * q + 0] = v.x;
+        if (4 * q + 1 < S) bnext[4 * q + 1] = v.y;
+        if (4 * q + 2 < S) bnext[4 * q + 2] = v.z;
+        if (4 * q + 3 < S) bnext[4 * q + 3] = v.w;
+      }
+      bcol = bp;
+    }
+
+    uint32_t dg[S], u[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      dg[i] = dtop[i];
+      u[i] = up[i];
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      uint32_t hn[S], dn[S];
+      if constexpr (CIRC == kExact) {
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn);
+      } else {
+        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
+      }
+      runmax<S, true>(M, dn, kill[r]);
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        dg[i] = H[r][i];
+        H[r][i] = hn[i];
+        u[i] = hn[i];
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < S; ++i) dtop[i] = up[i];
+    if (store_bnd) {  // my bottom row at this column, for the next stripe
+      uint4* d4 = reinterpret_cast<uint4*>(bnd + (int64_t(a.n) - 1 - cnt) * SP);
+#pragma unroll
+      for (int q = 0; q < SP / 4; ++q) {
+        uint4 v;
+        v.x = 4 * q + 0 < S ? H[R - 1][4 * q + 0] : 0u;
+        v.y = 4 * q + 1 < S ? H[R - 1][4 * q + 1] : 0u;
+        v.z = 4 * q + 2 < S ? H[R - 1][4 * q + 2] : 0u;
+        v.w = 4 * q + 3 < S ? H[R - 1][4 * q + 3] : 0u;
+        __stcg(d4 + q, v);
+      }
+    }
+    __syncwarp();  // orders the boundary store before lane 0's later load
+  }
+}
+
 template <int S, int R, int L, int CIRC, bool PAD, class K>
 void launch_sweep(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
   if constexpr (K::kFixed) {
     sw_sweep_kernel<S, R, L, CIRC, PAD, K><<<grid, block, 0, st>>>(a, K{});
   } else {
     sw_sweep_kernel<S, R, L, CIRC, PAD, KRun><<<grid, block, 0, st>>>(a, kr);
+  }
+}
+
+template <int S, int CIRC, class K>
+void launch_striped(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
+  if constexpr (K::kFixed) {
+    sw_sweep_striped_kernel<S, CIRC, K><<<grid, block, 0, st>>>(a, K{});
+  } else {
+    sw_sweep_striped_kernel<S, CIRC, KRun><<<grid, block, 0, st>>>(a, kr);
   }
 }
 
@@ -197,6 +393,17 @@ void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
 
 #define BPBC_CAT2(a, b) a##b
 #define BPBC_CAT(a, b) BPBC_CAT2(a, b)
+void BPBC_CAT(register_striped_s, BPBC_S)(SweepEntry (*tab)[13]) {
+  using K211 = KFix<2, 1, 1>;
+  tab[0][BPBC_S - 4] = {
+      &launch_striped<BPBC_S, kExact, K211>,
+      (const void*)&sw_sweep_striped_kernel<BPBC_S, kExact, K211>};
+  tab[1][BPBC_S - 4] = {&launch_striped<BPBC_S, kSat, K211>,
+                        (const void*)&sw_sweep_striped_kernel<BPBC_S, kSat, K211>};
+  tab[2][BPBC_S - 4] = {&launch_striped<BPBC_S, kSat, KRun>,
+                        (const void*)&sw_sweep_striped_kernel<BPBC_S, kSat, KRun>};
+}
+
 void BPBC_CAT(register_sweep_s, BPBC_S)(SweepEntry (*tab)[kNumRL][13]) {
   reg_rl<BPBC_S, 0, false>(tab);
   reg_rl<BPBC_S, 1, false>(tab);

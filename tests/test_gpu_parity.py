@@ -150,7 +150,7 @@ def test_errors():
     with pytest.raises(bpbc.BPBCError) as ei:
         bpbc.score_batch(q, t, 2, -1, -20, score_bits=4)
     assert ei.value.status == _lib.BPBC_ERR_INVALID_ARG
-    big = torch.zeros((4, 300), dtype=torch.uint8, device=DEV)
+    big = torch.zeros((4, (1 << 16) + 1), dtype=torch.uint8, device=DEV)  # > BPBC_MAX_QUERY_LEN
     with pytest.raises(bpbc.BPBCError) as ei:
         bpbc.score_batch(big, big)
     assert ei.value.status == _lib.BPBC_ERR_UNSUPPORTED
@@ -253,3 +253,41 @@ def test_multi_device_driver():
     q, t = synth.gen_pairs(2024, 3001, 64, 80, planted=True)
     got = parallel.score_multi_device(q, t, 2, -1, -1, 8, devices=[0, 0, 0])
     np.testing.assert_array_equal(got, oracle.sw_batch(q, t, 2, -1, -1, score_bits=8))
+
+
+# ---------------------------------------------------------------- long queries (striped kernel)
+
+
+@pytest.mark.parametrize("m,n", [(257, 257), (300, 300), (384, 520), (512, 512), (700, 1000),
+                                 (1000, 700), (129, 3000), (640, 640)])
+def test_long_query_lengths(m, n):
+    """min(m, n) > 256: 128-row stripes handed over through the boundary buffer."""
+    q, t = synth.gen_pairs(9000 + m * 7 + n, 100, m, n, planted=True)
+    check_full(q, t)
+    if min(m, n) > 256:
+        assert bpbc.last_plan(0)["rows_per_lane"] == 4
+
+
+@pytest.mark.parametrize("s", [6, 8, 10, 11, 12, 16])
+def test_c5_m512_width_sweep(s):
+    """C5's longest point (m = n = 512) at several widths: saturation law (R3)."""
+    q, t = synth.gen_pairs(synth.seed_for_config(5) + 512, 256, 512, 512, planted=True)
+    got = check_full(q, t, s=s)
+    exact = oracle.sw_batch(q, t, 2, -1, -1)
+    np.testing.assert_array_equal(got, np.minimum(exact, 2 ** s - 1))
+
+
+@pytest.mark.parametrize("consts", [(1, -1, -1), (3, -2, -1), (1, 0, 0), (5, -3, -4)])
+def test_long_query_runtime_constants(consts):
+    q, t = synth.gen_pairs(4321, 130, 300, 333, planted=True)
+    c1, mm, g = consts
+    check_full(q, t, c1, mm, g, 12)
+
+
+@pytest.mark.parametrize("s", [13, 14, 16])
+def test_m256_wide_width_uses_stripes(s):
+    """m in (128, 256] whose evaluated width is >= 13 bits (match = 31) goes to
+    the striped kernel (R = 8 rows x 13+ planes would spill)."""
+    q, t = synth.gen_pairs(777 + s, 200, 200, 240, planted=True)
+    check_full(q, t, 31, -1, -1, s=s)
+    assert bpbc.last_plan(0)["rows_per_lane"] == 4
