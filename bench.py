@@ -200,6 +200,9 @@ def main():
     ap.add_argument("--m", type=int, default=None, help="override the query length")
     ap.add_argument("--n", type=int, default=None, help="override the target length")
     ap.add_argument("--pairs", type=int, default=None, help="override the pair count")
+    ap.add_argument("--no-filter", action="store_true")
+    ap.add_argument("--filter-threshold", type=int, default=None,
+                    help="tau of the threshold-filter line (default 0.9 * min(m, n))")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
@@ -287,8 +290,40 @@ def main():
     cells = P_total * m * n * args.steps
     gcups = cells / (t_ms / 1e3) / 1e9
 
+    # ---------------- threshold filter (NEXT-2) on the same resident batch
+    filt = None
+    if not args.no_filter:
+        tau = args.filter_threshold if args.filter_threshold is not None else int(0.9 * min(m, n))
+        fmask = torch.empty((P + 31) // 32, dtype=torch.int32, device=dev)
+        fidx = torch.empty(P, dtype=torch.int64, device=dev)
+        fcnt = torch.zeros(1, dtype=torch.int64, device=dev)
+
+        def fstep():
+            bpbc.filter_batch(dq, dt, tau, *CONSTS, score_bits=s, workspace=ws)
+
+        for _ in range(args.warmup):
+            fstep()
+        fk = max(3, min(args.steps, 10))
+        fs = [torch.cuda.Event(enable_timing=True) for _ in range(fk)]
+        fe = [torch.cuda.Event(enable_timing=True) for _ in range(fk)]
+        torch.cuda.synchronize()
+        for k in range(fk):
+            flush.zero_()
+            fs[k].record()
+            fstep()
+            fe[k].record()
+        torch.cuda.synchronize()
+        f_ms = sum(x.elapsed_time(y) for x, y in zip(fs, fe))
+        _, cnt, _ = bpbc.filter_batch(dq, dt, tau, *CONSTS, score_bits=s, workspace=ws)
+        filt = {"value": round(P * m * n * fk / (f_ms / 1e3) / 1e9, 2), "unit": "GCUPS",
+                "threshold": tau, "flagged_pairs_rank0": int(cnt.item()),
+                "ms_per_step": round(f_ms / fk, 4),
+                "what": "bpbc_sw_filter_batch: pairs with max score > threshold, mask + "
+                        "ascending indices (P:L231)"}
+        del fmask, fidx, fcnt
+
     # ---------------- end to end through the host-buffer C call
-    e2e = None
+    e2e = e2e_packed2 = None
     if not args.no_e2e:
         hout = torch.empty(P, dtype=torch.int32, pin_memory=True)
         qn, tn, on = hq.numpy(), ht.numpy(), hout.numpy()
@@ -308,7 +343,32 @@ def main():
         e2e = {"value": round(P_total * m * n * ksteps / el / 1e9, 2), "unit": "GCUPS",
                "h2d_bytes_per_step": P_total * (m + n), "d2h_bytes_per_step": P_total * 4,
                "steps": ksteps, "timing": "host wall clock around the blocking C call "
-                                          "(pinned host buffers)"}
+                                          "bpbc_sw_score_batch_host (pinned host buffers, "
+                                          "1 byte per base)"}
+        # same through bpbc_sw_score_batch_host_packed2 (2-bit packed host
+        # rows, 4x fewer H2D bytes; packing is input preparation, untimed)
+        hq2 = torch.from_numpy(synth.pack2bit(hq.numpy())).pin_memory()
+        ht2 = torch.from_numpy(synth.pack2bit(ht.numpy())).pin_memory()
+        q2n, t2n = hq2.numpy(), ht2.numpy()
+        for _ in range(2):
+            bpbc.score_batch_host_packed2(q2n, t2n, m, n, *CONSTS, score_bits=s, device=local,
+                                          out=on)
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(ksteps):
+            bpbc.score_batch_host_packed2(q2n, t2n, m, n, *CONSTS, score_bits=s, device=local,
+                                          out=on)
+        el2 = time.perf_counter() - t0
+        if world > 1:
+            te = torch.tensor([el2], dtype=torch.float64, device=dev)
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+            el2 = te.item()
+        e2e_packed2 = {"value": round(P_total * m * n * ksteps / el2 / 1e9, 2), "unit": "GCUPS",
+                       "h2d_bytes_per_step": P_total * ((m + 3) // 4 + (n + 3) // 4),
+                       "d2h_bytes_per_step": P_total * 4, "steps": ksteps,
+                       "timing": "host wall clock around bpbc_sw_score_batch_host_packed2 "
+                                 "(pinned, 2-bit packed bases)"}
 
     # ---------------- result gather (outside the timed region) + parity sample
     if world > 1:  # rank r holds the pairs of shard_range(P_total, world, r)
@@ -376,7 +436,7 @@ def main():
                        "m": m, "n": n, "score_bits": s, "parallelism": f"dp{world} (pair shards)",
                        "l2": "inputs 320 MiB > 126 MB L2, plus a 256 MiB L2 flush between steps",
                        "plan": plan},
-            "e2e": e2e, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,
+            "e2e": e2e, "e2e_packed2": e2e_packed2, "filter": filt, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,
             # ours per step and rank: pack (query+target), sweep, extract
             "gpu_launches": 3 * args.steps * world, "parity": parity}
     print(json.dumps(line), flush=True)

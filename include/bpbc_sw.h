@@ -137,6 +137,51 @@ int bpbc_sw_score_batch_host(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8
                              int32_t *out_scores);
 
 /*
+ * Same as bpbc_sw_score_batch / bpbc_sw_score_batch_host with the bases
+ * 2-bit packed, 4 per byte (the paper's 2-bit code of P:L51, stored densely;
+ * SURVEY.md NEXT-1): row k of query2 is ceil(m/4) bytes and base i of it is
+ * bits [2(i%4), 2(i%4)+1] of byte i/4 (A=0, T=1, G=2, C=3; bits past the row
+ * end are ignored).  target2 likewise with ceil(n/4) bytes per row.  Cuts the
+ * input bytes (and the host->device copy of the _host variant) 4x; every code
+ * is valid, so BPBC_FLAG_BAD_BASE is never raised.  Rows are read with
+ * 16-byte loads when ceil(len/4) is a multiple of 16 and the buffer is 16-byte
+ * aligned, byte by byte otherwise.
+ */
+int bpbc_sw_score_batch_packed2(bpbc_sw_ctx *ctx, const uint8_t *query2, const uint8_t *target2,
+                                int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                                int32_t mismatch, int32_t gap, int32_t score_bits,
+                                int32_t *out_scores, void *workspace, size_t workspace_bytes,
+                                void *stream);
+int bpbc_sw_score_batch_host_packed2(bpbc_sw_ctx *ctx, const uint8_t *query2,
+                                     const uint8_t *target2, int64_t num_pairs, int32_t m,
+                                     int32_t n, int32_t match, int32_t mismatch, int32_t gap,
+                                     int32_t score_bits, int32_t *out_scores);
+
+/*
+ * Threshold filter (the paper's stated use: flag the pairs
+ * whose maximum score exceeds a threshold and re-align only those, with
+ * traceback, on the CPU).  Same hot path as bpbc_sw_score_batch with
+ * the per-cell running maximum (2s logic ops) replaced by a sticky
+ * "some cell > threshold" flag (s + 1 ops).
+ *
+ * threshold    0 <= threshold <= 2^score_bits - 2; a pair is flagged iff
+ *              its maximum local score > threshold.
+ * out_mask     device, uint32 [ceil(num_pairs/32)]: bit k of word g = flag of
+ *              pair 32g+k (bits past num_pairs are 0).  Required.
+ * out_indices  device, int64 [num_pairs] or NULL: the flagged pair indices in
+ *              ascending order (the first *out_count entries are written).
+ * out_count    device, int64 [1] or NULL: number of flagged pairs.
+ * The compaction uses ctx-owned scratch (grown on demand).  Other arguments
+ * and errors as bpbc_sw_score_batch; a threshold outside the range above is
+ * INVALID_ARG.  Asynchronous on `stream`.
+ */
+int bpbc_sw_filter_batch(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8_t *target,
+                         int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                         int32_t mismatch, int32_t gap, int32_t score_bits, int32_t threshold,
+                         uint32_t *out_mask, int64_t *out_indices, int64_t *out_count,
+                         void *workspace, size_t workspace_bytes, void *stream);
+
+/*
  * W2B step alone: bit-transpose base codes into planes.
  * codes   device, uint8 [num_pairs][len].
  * planes  device, uint32 [ceil(num_pairs/32)][len][2]: [g][i][0] = X^H_i,

@@ -35,6 +35,15 @@ SIGNATURES = {
     "bpbc_sw_score_batch_host": (_c.c_int, [_vp, _vp, _vp, _c.c_int64, _c.c_int32,
                                             _c.c_int32, _c.c_int32, _c.c_int32, _c.c_int32,
                                             _c.c_int32, _vp]),
+    "bpbc_sw_score_batch_packed2": (_c.c_int, [_vp, _vp, _vp, _c.c_int64, _c.c_int32,
+                                               _c.c_int32, _c.c_int32, _c.c_int32, _c.c_int32,
+                                               _c.c_int32, _vp, _vp, _c.c_size_t, _vp]),
+    "bpbc_sw_score_batch_host_packed2": (_c.c_int, [_vp, _vp, _vp, _c.c_int64, _c.c_int32,
+                                                    _c.c_int32, _c.c_int32, _c.c_int32,
+                                                    _c.c_int32, _c.c_int32, _vp]),
+    "bpbc_sw_filter_batch": (_c.c_int, [_vp, _vp, _vp, _c.c_int64, _c.c_int32, _c.c_int32,
+                                        _c.c_int32, _c.c_int32, _c.c_int32, _c.c_int32,
+                                        _c.c_int32, _vp, _vp, _vp, _vp, _c.c_size_t, _vp]),
     "bpbc_sw_pack": (_c.c_int, [_vp, _vp, _c.c_int64, _c.c_int32, _vp, _vp]),
     "bpbc_sw_untranspose": (_c.c_int, [_vp, _vp, _c.c_int64, _c.c_int32, _c.c_int32,
                                        _c.c_int64, _c.c_int32, _vp, _vp]),

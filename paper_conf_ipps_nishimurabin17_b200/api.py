@@ -107,6 +107,96 @@ def score_batch_host(query: np.ndarray, target: np.ndarray, match: int = 2, mism
     return out
 
 
+def filter_batch(query: torch.Tensor, target: torch.Tensor, threshold: int, match: int = 2,
+                 mismatch: int = -1, gap: int = -1, score_bits: int | None = None,
+                 indices: bool = True, workspace: torch.Tensor | None = None,
+                 stream=None):
+    """bpbc_sw_filter_batch: flag the pairs whose max local score > threshold
+    (the paper's filter use case).
+
+    Returns (mask, count, idx): mask int32 [ceil(P/32)] CUDA tensor of flag
+    words (bit k of word g = pair 32g+k; int32 view of the uint32 words),
+    count an int64 [1] CUDA tensor, idx an int64 [P] CUDA tensor whose first
+    count entries are the flagged pairs in ascending order (None if
+    indices=False)."""
+    if not (query.is_cuda and target.is_cuda):
+        raise ValueError("filter_batch needs CUDA tensors")
+    if query.dtype != torch.uint8 or target.dtype != torch.uint8:
+        raise TypeError("query/target must be uint8 base codes")
+    if query.dim() != 2 or target.dim() != 2 or query.shape[0] != target.shape[0]:
+        raise ValueError("query [P, m] and target [P, n] expected")
+    query, target = query.contiguous(), target.contiguous()
+    P, m = query.shape
+    n = target.shape[1]
+    dev = query.device.index if query.device.index is not None else torch.cuda.current_device()
+    if score_bits is None:
+        score_bits = default_score_bits(match, m, n)
+    mask = torch.empty((P + 31) // 32, dtype=torch.int32, device=query.device)
+    count = torch.zeros(1, dtype=torch.int64, device=query.device)
+    idx = torch.empty(P, dtype=torch.int64, device=query.device) if indices else None
+    ws_ptr, ws_bytes = None, 0
+    if workspace is not None:
+        ws_ptr, ws_bytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
+    ctx = _ctx(dev)
+    check(_lib.load().bpbc_sw_filter_batch(
+        ctx, query.data_ptr(), target.data_ptr(), P, m, n, match, mismatch, gap, score_bits,
+        threshold, mask.data_ptr(), idx.data_ptr() if idx is not None else None,
+        count.data_ptr(), ws_ptr, ws_bytes, _stream_ptr(stream, query.device)), ctx)
+    return mask, count, idx
+
+
+def score_batch_packed2(query2: torch.Tensor, target2: torch.Tensor, m: int, n: int,
+                        match: int = 2, mismatch: int = -1, gap: int = -1,
+                        score_bits: int | None = None, out: torch.Tensor | None = None,
+                        workspace: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """bpbc_sw_score_batch_packed2: query2 uint8 [P, ceil(m/4)], target2 uint8
+    [P, ceil(n/4)] CUDA tensors of 2-bit packed bases (4 per byte, base i in
+    bits 2(i%4) of byte i//4; include/bpbc_sw.h)."""
+    if not (query2.is_cuda and target2.is_cuda):
+        raise ValueError("score_batch_packed2 needs CUDA tensors")
+    if query2.dtype != torch.uint8 or target2.dtype != torch.uint8:
+        raise TypeError("packed rows must be uint8")
+    P = query2.shape[0]
+    if (query2.shape != (P, (m + 3) // 4) or target2.shape != (P, (n + 3) // 4)):
+        raise ValueError("query2 [P, ceil(m/4)] and target2 [P, ceil(n/4)] expected")
+    query2, target2 = query2.contiguous(), target2.contiguous()
+    dev = query2.device.index if query2.device.index is not None else torch.cuda.current_device()
+    if score_bits is None:
+        score_bits = default_score_bits(match, m, n)
+    if out is None:
+        out = torch.empty(P, dtype=torch.int32, device=query2.device)
+    ws_ptr, ws_bytes = None, 0
+    if workspace is not None:
+        ws_ptr, ws_bytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
+    ctx = _ctx(dev)
+    check(_lib.load().bpbc_sw_score_batch_packed2(
+        ctx, query2.data_ptr(), target2.data_ptr(), P, m, n, match, mismatch, gap, score_bits,
+        out.data_ptr(), ws_ptr, ws_bytes, _stream_ptr(stream, query2.device)), ctx)
+    return out
+
+
+def score_batch_host_packed2(query2: np.ndarray, target2: np.ndarray, m: int, n: int,
+                             match: int = 2, mismatch: int = -1, gap: int = -1,
+                             score_bits: int | None = None, device: int = 0,
+                             out: np.ndarray | None = None) -> np.ndarray:
+    """bpbc_sw_score_batch_host_packed2: host 2-bit packed rows in, host int32
+    scores out (blocking; 4x fewer host->device bytes than score_batch_host)."""
+    query2 = np.ascontiguousarray(query2, dtype=np.uint8)
+    target2 = np.ascontiguousarray(target2, dtype=np.uint8)
+    P = query2.shape[0]
+    if query2.shape != (P, (m + 3) // 4) or target2.shape != (P, (n + 3) // 4):
+        raise ValueError("query2 [P, ceil(m/4)] and target2 [P, ceil(n/4)] expected")
+    if score_bits is None:
+        score_bits = default_score_bits(match, m, n)
+    if out is None:
+        out = np.empty(P, dtype=np.int32)
+    ctx = _ctx(device)
+    check(_lib.load().bpbc_sw_score_batch_host_packed2(
+        ctx, query2.ctypes.data, target2.ctypes.data, P, m, n, match, mismatch, gap, score_bits,
+        out.ctypes.data), ctx)
+    return out
+
+
 def pack(codes: torch.Tensor, stream=None) -> torch.Tensor:
     """bpbc_sw_pack: uint8 [P, len] -> uint32 [ceil(P/32), len, 2] bit planes (H, L)."""
     codes = codes.contiguous()

@@ -25,6 +25,8 @@ struct bpbc_sw_ctx {
   // its own workspace, so chunk c+1's H2D overlaps chunk c's kernels
   cudaStream_t host_streams[2] = {nullptr, nullptr};
   void* ws_h[2] = {nullptr, nullptr};
+  void* fscratch = nullptr;  // filter compaction scratch (grown lazily)
+  size_t fscratch_bytes = 0;
   size_t ws_h_bytes[2] = {0, 0};
   char err[512] = {0};
   // last plan
@@ -51,39 +53,30 @@ struct bpbc_sw_ctx {
 namespace bpbc {
 namespace {
 
-SweepEntry g_table[kNumVariants][kNumRL][13];
-SweepEntry g_striped[3][13];
+SweepEntry g_table[2][kNumVariants][kNumRL][13];  // [mode][variant][rl][S - 4]
+SweepEntry g_striped[2][kNumStripeRV][3][13];     // [mode][stripe R][kind][S - 4]
 std::once_flag g_table_once;
 
 void init_table() {
   memset(g_table, 0, sizeof(g_table));
   memset(g_striped, 0, sizeof(g_striped));
-  register_striped_s4(g_striped);
-  register_striped_s5(g_striped);
-  register_striped_s6(g_striped);
-  register_striped_s7(g_striped);
-  register_striped_s8(g_striped);
-  register_striped_s9(g_striped);
-  register_striped_s10(g_striped);
-  register_striped_s11(g_striped);
-  register_striped_s12(g_striped);
-  register_striped_s13(g_striped);
-  register_striped_s14(g_striped);
-  register_striped_s15(g_striped);
-  register_striped_s16(g_striped);
-  register_sweep_s4(g_table);
-  register_sweep_s5(g_table);
-  register_sweep_s6(g_table);
-  register_sweep_s7(g_table);
-  register_sweep_s8(g_table);
-  register_sweep_s9(g_table);
-  register_sweep_s10(g_table);
-  register_sweep_s11(g_table);
-  register_sweep_s12(g_table);
-  register_sweep_s13(g_table);
-  register_sweep_s14(g_table);
-  register_sweep_s15(g_table);
-  register_sweep_s16(g_table);
+#define BPBC_REG(S)                                      \
+  register_sweep_s##S##_m0(g_table[0], g_striped[0]); \
+  register_sweep_s##S##_m1(g_table[1], g_striped[1]);
+  BPBC_REG(4)
+  BPBC_REG(5)
+  BPBC_REG(6)
+  BPBC_REG(7)
+  BPBC_REG(8)
+  BPBC_REG(9)
+  BPBC_REG(10)
+  BPBC_REG(11)
+  BPBC_REG(12)
+  BPBC_REG(13)
+  BPBC_REG(14)
+  BPBC_REG(15)
+  BPBC_REG(16)
+#undef BPBC_REG
 }
 
 int bit_length(int64_t v) {
@@ -115,7 +108,7 @@ Layout layout(int64_t P, int mq, int nt) {
   Layout L;
   L.G = (P + 31) / 32;
   // room for the striped kernel whenever the plan may pick it (m > 128)
-  L.stripes = mq > kStripeRows ? (mq + kStripeRows - 1) / kStripeRows : 1;
+  L.stripes = mq > 128 ? (mq + kMinStripeRows - 1) / kMinStripeRows : 1;
   const int64_t xbytes = (L.G * mq + kXBackPad) * 8;
   const int64_t ybytes = (kYFrontPad + L.G * nt + nt + kYBackPadExtra) * 8;
   const int64_t mpbytes = L.G * L.stripes * 32 * 16 * 4;
@@ -139,12 +132,24 @@ Layout layout(int64_t P, int mq, int nt) {
 
 struct Plan {
   int circuit, consts, rl, width, cap;
+  int stripe_rv = 1;  // striped kernels: index into kStripeRV
   bool pad;
   int ops;
 };
 
+// Rows per lane of the striped kernel: 4 unless BPBC_STRIPE_R=2 is set in the
+// environment (a tuning knob for benchmarks; read once).
+int stripe_rv_default() {
+  static const int rv = [] {
+    const char* v = getenv("BPBC_STRIPE_R");
+    return (v && atoi(v) == 2) ? 0 : 1;
+  }();
+  return rv;
+}
+
 // Choose the circuit, the evaluated width and the tiling.
 int make_plan(int mq, int c1, int c2, int g, int S, Plan* p) {
+  p->stripe_rv = stripe_rv_default();
   if (mq <= 32) p->rl = 0;
   else if (mq <= 64) p->rl = 1;
   else if (mq <= 128) p->rl = 2;
@@ -201,10 +206,80 @@ int validate_common(int64_t P, int m, int n, int match, int mismatch, int gap, i
   return BPBC_OK;
 }
 
-// Enqueue pack -> sweep -> extract on device buffers.
+// The sweep kernel a plan runs and how many group streams fit on the device.
+struct Dispatch {
+  Plan plan;
+  SweepEntry ent;
+  bool striped;
+  int R, L;
+  int64_t cap_streams;  // resident streams (before the boundary-buffer cap)
+};
+
+// Cap on resident sweep blocks per SM: BPBC_MAX_BLOCKS_PER_SM in the
+// environment (tuning knob for benchmarks; read once), else none.
+int max_blocks_env() {
+  static const int v = [] {
+    const char* e = getenv("BPBC_MAX_BLOCKS_PER_SM");
+    return e ? atoi(e) : 0;
+  }();
+  return v;
+}
+
+int occupancy_blocks(const void* func) {  // cached per kernel
+  static std::mutex mu;
+  static std::vector<std::pair<const void*, int>> cache;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    for (auto& kv : cache)
+      if (kv.first == func) return kv.second;
+  }
+  int nb = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, func, 128, 0) != cudaSuccess) return -1;
+  if (nb < 1) nb = 1;
+  std::lock_guard<std::mutex> lk(mu);
+  cache.emplace_back(func, nb);
+  return nb;
+}
+
+int make_dispatch(bpbc_sw_ctx* ctx, int mq, int c1, int c2, int g, int S, Dispatch* d,
+                  int mode = kModeMax) {
+  int rc = make_plan(mq, c1, c2, g, S, &d->plan);
+  if (rc != BPBC_OK) return rc;
+  std::call_once(g_table_once, init_table);
+  const Plan& plan = d->plan;
+  d->striped = plan.rl < 0;
+  d->ent = d->striped
+               ? g_striped[mode][plan.stripe_rv]
+                          [plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]
+                          [plan.width - 4]
+               : g_table[mode][variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl]
+                        [plan.width - 4];
+  if (!d->ent.launch) return BPBC_ERR_UNSUPPORTED;
+  d->R = d->striped ? kStripeRV[plan.stripe_rv] : kRLR[plan.rl];
+  d->L = d->striped ? 32 : kRLL[plan.rl];
+  int nb = occupancy_blocks(d->ent.func);
+  if (nb < 0) return cuda_fail(ctx, cudaGetLastError(), "occupancy");
+  if (max_blocks_env() > 0 && nb > max_blocks_env()) nb = max_blocks_env();
+  d->cap_streams = int64_t(ctx->num_sms) * nb * 4 * (32 / d->L);
+  return BPBC_OK;
+}
+
+// What the sweep produces: max scores (extract) or threshold flags (filter).
+struct RunOut {
+  int32_t* scores = nullptr;     // max mode
+  int mode = kModeMax;
+  int threshold = 0;             // threshold mode: flag pairs with score > threshold
+  uint32_t* mask = nullptr;      //   [ceil(P/32)] flag words
+  int64_t* indices = nullptr;    //   optional ascending flagged pair indices
+  int64_t* count = nullptr;      //   optional number of flagged pairs
+  void* scratch = nullptr;       //   compaction scratch (filter_scratch_bytes)
+  size_t scratch_bytes = 0;
+};
+
+// Enqueue pack -> sweep -> extract (or the filter epilogue) on device buffers.
 int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, int64_t P, int m,
-               int n, int match, int mismatch, int gap, int S, int32_t* out, uint8_t* ws,
-               cudaStream_t st) {
+               int n, int match, int mismatch, int gap, int S, const RunOut& o, uint8_t* ws,
+               cudaStream_t st, bool packed2) {
   // score is symmetric (R17): the shorter sequence plays the query (rows)
   const uint8_t* qx = query;
   const uint8_t* ty = target;
@@ -216,9 +291,10 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
     nt = m;
   }
   const int c1 = match, c2 = -mismatch, g = -gap;
-  Plan plan;
-  int rc = make_plan(mq, c1, c2, g, S, &plan);
+  Dispatch dsp;
+  int rc = make_dispatch(ctx, mq, c1, c2, g, S, &dsp, o.mode);
   if (rc != BPBC_OK) return rc;
+  const Plan& plan = dsp.plan;
   const Layout lay = layout(P, mq, nt);
   uint2* Xp = reinterpret_cast<uint2*>(ws + lay.x_off);
   uint2* Ybase = reinterpret_cast<uint2*>(ws + lay.y_off);
@@ -229,25 +305,16 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   if (ctx->profiling)
     for (int i = 0; i < 4; ++i) ev[i] = ctx->take_event();
   if (ev[0]) cudaEventRecord(ev[0], st);
-  cudaError_t e = launch_pack2(qx, mq, Xp, ty, nt, Yp, P, ctx->d_flags, ctx->num_sms, st);
+  cudaError_t e =
+      launch_pack2(qx, mq, Xp, ty, nt, Yp, P, ctx->d_flags, ctx->num_sms, st, packed2);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "pack");
 
   if (ev[1]) cudaEventRecord(ev[1], st);
-  std::call_once(g_table_once, init_table);
-  const bool striped = plan.rl < 0;
-  const SweepEntry ent =
-      striped ? g_striped[plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]
-                         [plan.width - 4]
-              : g_table[variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl]
-                       [plan.width - 4];
-  if (!ent.launch) return BPBC_ERR_UNSUPPORTED;
-  const int R = striped ? kStripeR : kRLR[plan.rl], L = striped ? 32 : kRLL[plan.rl];
-  int nb = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, ent.func, 128, 0);
-  if (e != cudaSuccess) return cuda_fail(ctx, e, "occupancy");
-  if (nb < 1) nb = 1;
+  const bool striped = dsp.striped;
+  const SweepEntry ent = dsp.ent;
+  const int R = dsp.R, L = dsp.L;
   const int64_t segs = 32 / L;
-  int64_t cap_streams = int64_t(ctx->num_sms) * nb * 4 * segs;
+  int64_t cap_streams = dsp.cap_streams;
   if (striped && cap_streams > lay.bnd_streams) cap_streams = lay.bnd_streams;
   SweepArgs a;
   a.Xp = Xp;
@@ -256,13 +323,34 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   a.G = lay.G;
   a.m = mq;
   a.n = nt;
-  a.streams = lay.G < cap_streams ? lay.G : cap_streams;
+  // Streams come in whole blocks on every SM (4 warps x 32/L streams per
+  // block, b blocks per SM).  The SMs are ALU-bound, so an SM's time is its
+  // total work: b * 4 * segs * ceil(G / streams) groups.  Pick b in
+  // [nb - 1, nb] minimising that (ties -> more warps for latency hiding);
+  // the streams then split the groups as evenly as possible (base / rem).
+  {
+    const int64_t per_block = 4 * segs;
+    const int64_t nb = cap_streams / (int64_t(ctx->num_sms) * per_block);
+    int64_t best_b = nb > 0 ? nb : 1, best_t = -1;
+    for (int64_t b = nb; b >= 1 && b >= nb - 1; --b) {
+      const int64_t st_b = int64_t(ctx->num_sms) * b * per_block;
+      const int64_t t = b * per_block * ((lay.G + st_b - 1) / st_b);
+      if (best_t < 0 || t < best_t) {
+        best_t = t;
+        best_b = b;
+      }
+    }
+    int64_t cap_b = int64_t(ctx->num_sms) * best_b * per_block;
+    if (nb < 1 || cap_b > cap_streams) cap_b = cap_streams;  // boundary-buffer cap
+    a.streams = lay.G < cap_b ? lay.G : cap_b;
+  }
   a.base = lay.G / a.streams;
   a.rem = lay.G % a.streams;
-  a.stripes = striped ? (mq + kStripeRows - 1) / kStripeRows : 1;
+  a.stripes = striped ? (mq + 32 * R - 1) / (32 * R) : 1;
   a.bnd = reinterpret_cast<uint32_t*>(ws + lay.bnd_off);
   a.bzero = reinterpret_cast<const uint32_t*>(ws + lay.zero_off);
   a.steps = (a.base + (a.rem > 0 ? 1 : 0)) * a.stripes * int64_t(nt) + L;
+  a.steps += a.steps & 1;  // the short kernel runs two steps per iteration
   if (striped) {
     e = cudaMemsetAsync(ws + lay.zero_off, 0, 256, st);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "memset(zero row)");
@@ -278,12 +366,22 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
     kr.gmask[i] = (g >> i) & 1 ? 0xFFFFFFFFu : 0u;
   }
   kr.zmask = c2 == 0 ? 0xFFFFFFFFu : 0u;
+  // threshold mode compares the diagonal term with tau (+ g for the exact
+  // circuit, whose D' carries the offset g)
+  const int tcmp = o.threshold + (plan.circuit == kExact ? g : 0);
+  for (int i = 0; i < 16; ++i) a.tmask[i] = (tcmp >> i) & 1 ? 0xFFFFFFFFu : 0u;
   ent.launch(a, kr, grid, 128, st);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(ctx, e, "sweep");
   if (ev[2]) cudaEventRecord(ev[2], st);
-  e = launch_extract(Mpart, lay.G, L * a.stripes, W, P, plan.cap, out, ctx->num_sms, st);
-  if (e != cudaSuccess) return cuda_fail(ctx, e, "extract");
+  if (o.mode == kModeThreshold) {
+    e = launch_filter_finish(Mpart, lay.G, L * a.stripes, P, o.mask, o.indices, o.count,
+                             o.scratch, o.scratch_bytes, ctx->num_sms, st);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "filter epilogue");
+  } else {
+    e = launch_extract(Mpart, lay.G, L * a.stripes, W, P, plan.cap, o.scores, ctx->num_sms, st);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "extract");
+  }
   if (ev[3]) cudaEventRecord(ev[3], st);
 
   ctx->plan_circuit = plan.circuit;
@@ -340,6 +438,124 @@ struct DeviceGuard {
 
 using namespace bpbc;
 
+namespace {
+
+int score_batch_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target,
+                        int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                        int32_t mismatch, int32_t gap, int32_t score_bits, int32_t* out_scores,
+                        void* workspace, size_t workspace_bytes, void* stream, bool packed2) {
+  if (!ctx) return BPBC_ERR_INVALID_ARG;
+  int rc = validate_common(num_pairs, m, n, match, mismatch, gap, score_bits);
+  if (rc != BPBC_OK) return rc;
+  if (num_pairs == 0) return BPBC_OK;
+  if (!query || !target || !out_scores) return BPBC_ERR_INVALID_ARG;
+  size_t need = 0;
+  bpbc_sw_workspace_bytes(num_pairs, m, n, &need);
+  DeviceGuard dg(ctx->device);
+  uint8_t* ws;
+  if (workspace) {
+    if (workspace_bytes < need) return BPBC_ERR_INVALID_ARG;
+    ws = static_cast<uint8_t*>(workspace);
+  } else {
+    rc = ensure_ws(ctx, need);
+    if (rc != BPBC_OK) return rc;
+    ws = static_cast<uint8_t*>(ctx->ws);
+  }
+  RunOut o;
+  o.scores = out_scores;
+  return run_device(ctx, query, target, num_pairs, m, n, match, mismatch, gap, score_bits, o, ws,
+                    static_cast<cudaStream_t>(stream), packed2);
+}
+
+int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target,
+                             int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                             int32_t mismatch, int32_t gap, int32_t score_bits,
+                             int32_t* out_scores, bool packed2) {
+  if (!ctx) return BPBC_ERR_INVALID_ARG;
+  int rc = validate_common(num_pairs, m, n, match, mismatch, gap, score_bits);
+  if (rc != BPBC_OK) return rc;
+  if (num_pairs == 0) return BPBC_OK;
+  if (!query || !target || !out_scores) return BPBC_ERR_INVALID_ARG;
+  DeviceGuard dg(ctx->device);
+  cudaError_t e;
+  for (int i = 0; i < 2; ++i) {
+    if (!ctx->host_streams[i]) {
+      e = cudaStreamCreateWithFlags(&ctx->host_streams[i], cudaStreamNonBlocking);
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaStreamCreate");
+    }
+  }
+  // bytes per row: one per base, or 4 bases per byte (packed2)
+  const int64_t qs = packed2 ? (int64_t(m) + 3) / 4 : m, ts = packed2 ? (int64_t(n) + 3) / 4 : n;
+  const size_t qb = size_t(num_pairs) * qs, tb = size_t(num_pairs) * ts,
+               ob = size_t(num_pairs) * sizeof(int32_t);
+  // Chunks in whole "waves" (one group per resident sweep stream, so every
+  // stream of a chunk gets the same number of groups), growing 1, 2, 4, ...
+  // waves: the first copy is short, later chunks amortise the pipeline fill.
+  Dispatch dsp;
+  rc = make_dispatch(ctx, m < n ? m : n, match, -mismatch, -gap, score_bits, &dsp);
+  if (rc != BPBC_OK) return rc;
+  const int64_t wave_pairs = dsp.cap_streams * 32;
+  // copy-bound (u8 rows: ~1 byte per base vs ~50 GB/s H2D) -> equal chunks so
+  // the last chunk's kernels are short; compute-bound (packed2) -> growing
+  // chunks so the first copy is short.  Estimate: H2D s/pair vs sweep s/pair.
+  const double h2d_s = double(qs + ts) / 50e9, sweep_s = double(m) * n / 5e12;
+  std::vector<int64_t> bounds{0};
+  if (h2d_s >= sweep_s) {
+    const int64_t waves = (num_pairs + wave_pairs - 1) / wave_pairs;
+    const int64_t per = (waves + 7) / 8;  // about 8 chunks of whole waves
+    while (bounds.back() < num_pairs) {
+      const int64_t left = num_pairs - bounds.back();
+      bounds.push_back(bounds.back() + (left < per * wave_pairs ? left : per * wave_pairs));
+    }
+  } else {
+    for (int64_t w = 1; bounds.back() < num_pairs; w = w < 8 ? 2 * w : 8) {
+      const int64_t left = num_pairs - bounds.back();
+      // fold a short remainder (< 1 wave) into this chunk
+      const int64_t take = left <= (w + 1) * wave_pairs ? left : w * wave_pairs;
+      bounds.push_back(bounds.back() + take);
+    }
+  }
+  int64_t chunk = 0;
+  for (size_t i = 1; i < bounds.size(); ++i)
+    chunk = bounds[i] - bounds[i - 1] > chunk ? bounds[i] - bounds[i - 1] : chunk;
+  size_t need = 0;
+  bpbc_sw_workspace_bytes(chunk, m, n, &need);
+  if ((rc = grow(ctx, (void**)&ctx->d_q, &ctx->d_q_bytes, qb, "cudaMalloc(q)")) != BPBC_OK) return rc;
+  if ((rc = grow(ctx, (void**)&ctx->d_t, &ctx->d_t_bytes, tb, "cudaMalloc(t)")) != BPBC_OK) return rc;
+  if ((rc = grow(ctx, (void**)&ctx->d_out, &ctx->d_out_bytes, ob, "cudaMalloc(out)")) != BPBC_OK)
+    return rc;
+  for (int i = 0; i < 2; ++i)
+    if ((rc = grow(ctx, &ctx->ws_h[i], &ctx->ws_h_bytes[i], need, "cudaMalloc(workspace)")) !=
+        BPBC_OK)
+      return rc;
+  for (size_t ci = 0; ci + 1 < bounds.size(); ++ci) {
+    const int64_t c0 = bounds[ci], cp = bounds[ci + 1] - bounds[ci];
+    cudaStream_t st = ctx->host_streams[ci & 1];
+    e = cudaMemcpyAsync(ctx->d_q + c0 * qs, query + c0 * qs, size_t(cp * qs),
+                        cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(ctx->d_t + c0 * ts, target + c0 * ts, size_t(cp * ts),
+                          cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "H2D");
+    RunOut o;
+    o.scores = ctx->d_out + c0;
+    rc = run_device(ctx, ctx->d_q + c0 * qs, ctx->d_t + c0 * ts, cp, m, n, match, mismatch, gap,
+                    score_bits, o, static_cast<uint8_t*>(ctx->ws_h[ci & 1]), st, packed2);
+    if (rc != BPBC_OK) return rc;
+    e = cudaMemcpyAsync(out_scores + c0, ctx->d_out + c0, size_t(cp) * sizeof(int32_t),
+                        cudaMemcpyDeviceToHost, st);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "D2H");
+  }
+  for (int i = 0; i < 2; ++i) {
+    e = cudaStreamSynchronize(ctx->host_streams[i]);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "sync");
+  }
+  return BPBC_OK;
+}
+
+}  // namespace
+
+
 extern "C" {
 
 const char* bpbc_sw_status_string(int status) {
@@ -392,6 +608,7 @@ int bpbc_sw_destroy(bpbc_sw_ctx* ctx) {
     if (ctx->host_streams[i]) cudaStreamDestroy(ctx->host_streams[i]);
     if (ctx->ws_h[i]) cudaFree(ctx->ws_h[i]);
   }
+  if (ctx->fscratch) cudaFree(ctx->fscratch);
   for (cudaEvent_t e : ctx->ev_pool) cudaEventDestroy(e);
   delete ctx;
   return BPBC_OK;
@@ -409,14 +626,34 @@ int bpbc_sw_score_batch(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* t
                         int64_t num_pairs, int32_t m, int32_t n, int32_t match,
                         int32_t mismatch, int32_t gap, int32_t score_bits, int32_t* out_scores,
                         void* workspace, size_t workspace_bytes, void* stream) {
+  return score_batch_impl(ctx, query, target, num_pairs, m, n, match, mismatch, gap, score_bits,
+                          out_scores, workspace, workspace_bytes, stream, false);
+}
+
+int bpbc_sw_filter_batch(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target,
+                         int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                         int32_t mismatch, int32_t gap, int32_t score_bits, int32_t threshold,
+                         uint32_t* out_mask, int64_t* out_indices, int64_t* out_count,
+                         void* workspace, size_t workspace_bytes, void* stream) {
   if (!ctx) return BPBC_ERR_INVALID_ARG;
   int rc = validate_common(num_pairs, m, n, match, mismatch, gap, score_bits);
   if (rc != BPBC_OK) return rc;
+  // "score > threshold" is decidable at width s only below the cap (R3)
+  if (threshold < 0 || int64_t(threshold) > (int64_t(1) << score_bits) - 2)
+    return BPBC_ERR_INVALID_ARG;
   if (num_pairs == 0) return BPBC_OK;
-  if (!query || !target || !out_scores) return BPBC_ERR_INVALID_ARG;
+  if (!query || !target || !out_mask) return BPBC_ERR_INVALID_ARG;
+  DeviceGuard dg(ctx->device);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const int64_t G = (num_pairs + 31) / 32;
+  const int mq = m < n ? m : n;
+  if (int64_t(threshold) >= int64_t(match) * mq) {  // no local alignment can exceed it
+    cudaError_t e = cudaMemsetAsync(out_mask, 0, size_t(G) * 4, st);
+    if (e == cudaSuccess && out_count) e = cudaMemsetAsync(out_count, 0, 8, st);
+    return e == cudaSuccess ? BPBC_OK : cuda_fail(ctx, e, "memset");
+  }
   size_t need = 0;
   bpbc_sw_workspace_bytes(num_pairs, m, n, &need);
-  DeviceGuard dg(ctx->device);
   uint8_t* ws;
   if (workspace) {
     if (workspace_bytes < need) return BPBC_ERR_INVALID_ARG;
@@ -426,66 +663,46 @@ int bpbc_sw_score_batch(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* t
     if (rc != BPBC_OK) return rc;
     ws = static_cast<uint8_t*>(ctx->ws);
   }
-  return run_device(ctx, query, target, num_pairs, m, n, match, mismatch, gap, score_bits,
-                    out_scores, ws, static_cast<cudaStream_t>(stream));
+  RunOut o;
+  o.mode = kModeThreshold;
+  o.threshold = threshold;
+  o.mask = out_mask;
+  o.indices = out_indices;
+  o.count = out_count;
+  if (out_indices || out_count) {
+    rc = grow(ctx, &ctx->fscratch, &ctx->fscratch_bytes, filter_scratch_bytes(G),
+              "cudaMalloc(filter scratch)");
+    if (rc != BPBC_OK) return rc;
+    o.scratch = ctx->fscratch;
+    o.scratch_bytes = ctx->fscratch_bytes;
+  }
+  return run_device(ctx, query, target, num_pairs, m, n, match, mismatch, gap, score_bits, o, ws,
+                    st, false);
+}
+
+int bpbc_sw_score_batch_packed2(bpbc_sw_ctx* ctx, const uint8_t* query2, const uint8_t* target2,
+                                int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                                int32_t mismatch, int32_t gap, int32_t score_bits,
+                                int32_t* out_scores, void* workspace, size_t workspace_bytes,
+                                void* stream) {
+  return score_batch_impl(ctx, query2, target2, num_pairs, m, n, match, mismatch, gap,
+                          score_bits, out_scores, workspace, workspace_bytes, stream, true);
 }
 
 int bpbc_sw_score_batch_host(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target,
                              int64_t num_pairs, int32_t m, int32_t n, int32_t match,
                              int32_t mismatch, int32_t gap, int32_t score_bits,
                              int32_t* out_scores) {
-  if (!ctx) return BPBC_ERR_INVALID_ARG;
-  int rc = validate_common(num_pairs, m, n, match, mismatch, gap, score_bits);
-  if (rc != BPBC_OK) return rc;
-  if (num_pairs == 0) return BPBC_OK;
-  if (!query || !target || !out_scores) return BPBC_ERR_INVALID_ARG;
-  DeviceGuard dg(ctx->device);
-  cudaError_t e;
-  for (int i = 0; i < 2; ++i) {
-    if (!ctx->host_streams[i]) {
-      e = cudaStreamCreateWithFlags(&ctx->host_streams[i], cudaStreamNonBlocking);
-      if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaStreamCreate");
-    }
-  }
-  const size_t qb = size_t(num_pairs) * m, tb = size_t(num_pairs) * n,
-               ob = size_t(num_pairs) * sizeof(int32_t);
-  // chunks of >= 64K pairs (multiples of 32), at most 8
-  int64_t nchunks = (num_pairs + 65535) / 65536;
-  if (nchunks > 8) nchunks = 8;
-  if (nchunks < 1) nchunks = 1;
-  int64_t chunk = (num_pairs + nchunks - 1) / nchunks;
-  chunk = (chunk + 31) / 32 * 32;
-  size_t need = 0;
-  bpbc_sw_workspace_bytes(chunk < num_pairs ? chunk : num_pairs, m, n, &need);
-  if ((rc = grow(ctx, (void**)&ctx->d_q, &ctx->d_q_bytes, qb, "cudaMalloc(q)")) != BPBC_OK) return rc;
-  if ((rc = grow(ctx, (void**)&ctx->d_t, &ctx->d_t_bytes, tb, "cudaMalloc(t)")) != BPBC_OK) return rc;
-  if ((rc = grow(ctx, (void**)&ctx->d_out, &ctx->d_out_bytes, ob, "cudaMalloc(out)")) != BPBC_OK)
-    return rc;
-  for (int i = 0; i < 2; ++i)
-    if ((rc = grow(ctx, &ctx->ws_h[i], &ctx->ws_h_bytes[i], need, "cudaMalloc(workspace)")) !=
-        BPBC_OK)
-      return rc;
-  for (int64_t c0 = 0, ci = 0; c0 < num_pairs; c0 += chunk, ++ci) {
-    const int64_t cp = num_pairs - c0 < chunk ? num_pairs - c0 : chunk;
-    cudaStream_t st = ctx->host_streams[ci & 1];
-    e = cudaMemcpyAsync(ctx->d_q + c0 * m, query + c0 * m, size_t(cp) * m,
-                        cudaMemcpyHostToDevice, st);
-    if (e == cudaSuccess)
-      e = cudaMemcpyAsync(ctx->d_t + c0 * n, target + c0 * n, size_t(cp) * n,
-                          cudaMemcpyHostToDevice, st);
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "H2D");
-    rc = run_device(ctx, ctx->d_q + c0 * m, ctx->d_t + c0 * n, cp, m, n, match, mismatch, gap,
-                    score_bits, ctx->d_out + c0, static_cast<uint8_t*>(ctx->ws_h[ci & 1]), st);
-    if (rc != BPBC_OK) return rc;
-    e = cudaMemcpyAsync(out_scores + c0, ctx->d_out + c0, size_t(cp) * sizeof(int32_t),
-                        cudaMemcpyDeviceToHost, st);
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "D2H");
-  }
-  for (int i = 0; i < 2; ++i) {
-    e = cudaStreamSynchronize(ctx->host_streams[i]);
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "sync");
-  }
-  return BPBC_OK;
+  return score_batch_host_impl(ctx, query, target, num_pairs, m, n, match, mismatch, gap,
+                               score_bits, out_scores, false);
+}
+
+int bpbc_sw_score_batch_host_packed2(bpbc_sw_ctx* ctx, const uint8_t* query2,
+                                     const uint8_t* target2, int64_t num_pairs, int32_t m,
+                                     int32_t n, int32_t match, int32_t mismatch, int32_t gap,
+                                     int32_t score_bits, int32_t* out_scores) {
+  return score_batch_host_impl(ctx, query2, target2, num_pairs, m, n, match, mismatch, gap,
+                               score_bits, out_scores, true);
 }
 
 int bpbc_sw_pack(bpbc_sw_ctx* ctx, const uint8_t* codes, int64_t num_pairs, int32_t len,

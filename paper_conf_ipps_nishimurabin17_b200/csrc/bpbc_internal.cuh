@@ -17,6 +17,7 @@ constexpr int64_t kXBackPad = 512;   // uint2 words after the last X group
 constexpr int64_t kYBackPadExtra = 128;
 
 enum Circuit : int { kExact = 0, kSat = 1 };
+enum Mode : int { kModeMax = 0, kModeThreshold = 1 };  // running max / sticky flag
 enum Consts : int { kC211 = 0, kCRun = 1 };
 constexpr int kNumVariants = 8;  // circuit x consts x padded-rows
 constexpr int variant_index(int circuit, int consts, bool pad) {
@@ -35,14 +36,18 @@ struct SweepArgs {
   int64_t rem;       //   (the first rem streams get base+1)
   int64_t steps;     // wavefront steps = (base + (rem>0)) * stripes * n + L
   // long-query (striped) kernel only
+  // threshold mode (bpbc_sw_filter_batch): bits of the compared threshold as
+  // all-ones / all-zeros masks (tau + g for the exact circuit, tau otherwise)
+  uint32_t tmask[16];
   int stripes;          // row stripes of kStripeRows per group (1 = short kernel)
   uint32_t* bnd;        // [streams][n][SP] stripe boundary rows
   const uint32_t* bzero;  // 16 zero words
 };
 
-// Long queries: stripes of kStripeR rows per lane x 32 lanes.
-constexpr int kStripeR = 4;
-constexpr int kStripeRows = 32 * kStripeR;
+// Long queries: stripes of R rows per lane x 32 lanes, R in kStripeRV.
+constexpr int kNumStripeRV = 2;
+constexpr int kStripeRV[kNumStripeRV] = {2, 4};
+constexpr int kMinStripeRows = 64;  // workspace is sized for the smallest stripes
 constexpr int kMaxShortRows = 256;     // m <= 256: the short kernel
 constexpr int64_t kMaxStripeStreams = 4096;
 constexpr int64_t kMaxBoundaryBytes = int64_t(1) << 30;
@@ -60,8 +65,13 @@ struct SweepEntry {
 };
 SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
 
-// Registration hooks, one per score width (sweep.cu compiled once per S).
-#define BPBC_DECLARE_REG(S) void register_sweep_s##S(SweepEntry (*tab)[kNumRL][13]);
+// Registration hooks, one per (score width, mode): sweep.cu is compiled once
+// per pair with -DBPBC_S=S -DBPBC_MODE=M.  tab: [variant][rl][S-4] of the
+// short kernel, stab: [stripe R variant][striped kind][S-4] (0 exact (+2,-1,-1), 1 saturating
+// (+2,-1,-1), 2 saturating runtime constants).
+#define BPBC_DECLARE_REG(S)                                                       \
+  void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13]); \
+  void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13]);
 BPBC_DECLARE_REG(4)
 BPBC_DECLARE_REG(5)
 BPBC_DECLARE_REG(6)
@@ -76,31 +86,21 @@ BPBC_DECLARE_REG(14)
 BPBC_DECLARE_REG(15)
 BPBC_DECLARE_REG(16)
 #undef BPBC_DECLARE_REG
-// Striped kernels: [0] exact (+2,-1,-1), [1] saturating (+2,-1,-1),
-// [2] saturating runtime constants; index S - 4.
-#define BPBC_DECLARE_SREG(S) void register_striped_s##S(SweepEntry (*tab)[13]);
-BPBC_DECLARE_SREG(4)
-BPBC_DECLARE_SREG(5)
-BPBC_DECLARE_SREG(6)
-BPBC_DECLARE_SREG(7)
-BPBC_DECLARE_SREG(8)
-BPBC_DECLARE_SREG(9)
-BPBC_DECLARE_SREG(10)
-BPBC_DECLARE_SREG(11)
-BPBC_DECLARE_SREG(12)
-BPBC_DECLARE_SREG(13)
-BPBC_DECLARE_SREG(14)
-BPBC_DECLARE_SREG(15)
-BPBC_DECLARE_SREG(16)
-#undef BPBC_DECLARE_SREG
 
 // pack.cu: one launch packs up to two [num_pairs][len] code arrays (query and
 // target); a job with codes == nullptr is skipped.
 cudaError_t launch_pack2(const uint8_t* codes_a, int len_a, uint2* planes_a,
                          const uint8_t* codes_b, int len_b, uint2* planes_b, int64_t num_pairs,
-                         uint32_t* flags, int num_sms, cudaStream_t stream);
+                         uint32_t* flags, int num_sms, cudaStream_t stream,
+                         bool packed2 = false);
 cudaError_t launch_pack(const uint8_t* codes, int64_t num_pairs, int len, uint2* planes,
                         uint32_t* flags, int num_sms, cudaStream_t stream);
+// filter.cu: threshold-mode epilogue (mask words, ascending indices, count)
+size_t filter_scratch_bytes(int64_t num_groups);
+cudaError_t launch_filter_finish(const uint32_t* partial, int64_t num_groups, int lanes,
+                                 int64_t num_pairs, uint32_t* mask, int64_t* indices,
+                                 int64_t* count, void* scratch, size_t scratch_bytes,
+                                 int num_sms, cudaStream_t stream);
 // extract.cu
 cudaError_t launch_extract(const uint32_t* partial, int64_t num_groups, int lanes, int s,
                            int64_t num_pairs, int32_t cap, int32_t* out, int num_sms,

@@ -139,6 +139,23 @@ BPBC_HD void runmax(uint32_t (&M)[S], const uint32_t (&H)[S], uint32_t kill) {
   mux<S>(p, M, H, M);
 }
 
+// Threshold filter (NEXT-2, the paper's use case P:L231): sticky flag
+// F |= (D > T) over lanes whose kill bit is 0.  T's bits come as all-ones /
+// all-zeros masks tm[i] (kernel parameters, read from the constant bank by
+// the gates).  The borrow out of T - D is lt(T, D) (S LOP3); + 1 to fold it
+// into F.  Replaces the 2S-LOP3 running max when only "score > T" is needed.
+template <int S, bool KILL>
+BPBC_HD void flag_gt(uint32_t& F, const uint32_t (&D)[S], const uint32_t* tm, uint32_t kill) {
+  uint32_t p = lop3<kNaAndB>(tm[0], D[0], 0u);
+#pragma unroll
+  for (int i = 1; i < S; ++i) p = lop3<kMajNa>(tm[i], D[i], p);
+  if constexpr (KILL) {
+    F = lop3<T8(TA | (TB & ~TC))>(F, p, kill);
+  } else {
+    F = lop3<T8(TA | TB)>(F, p, 0u);
+  }
+}
+
 // e = (xH ^ yH) | (xL ^ yL): 1 where the 2-bit bases differ.
 BPBC_HD uint32_t mismatch_flag(uint32_t xh, uint32_t xl, uint32_t yh, uint32_t yl) {
   return lop3<kOrXor>(lop3<kXor2>(xh, yh, 0u), xl, yl);

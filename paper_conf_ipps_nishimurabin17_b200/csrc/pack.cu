@@ -44,13 +44,20 @@ __device__ __forceinline__ int pos_of_bit(int i) {
   return (i & 1) ? 4 * q + b : 16 + 4 * q + b;
 }
 
+// Position held by bit i for 2-bit packed input (base i of a row in bits
+// 2i, 2i+1 of its little-endian words): H takes word A's odd bits (positions
+// 0..15) and word B's odd bits shifted to the even slots (16..31).
+__device__ __forceinline__ int pos_of_bit_packed2(int i) { return (i & 1) ? (i >> 1) : 16 + (i >> 1); }
+
 struct PackJob {
-  const uint8_t* codes;  // [num_pairs][len]
+  const uint8_t* codes;  // [num_pairs][stride]: u8 codes, or 2-bit packed
   uint2* planes;         // [G][len]
   int len;
+  int64_t stride;        // bytes per row: len (u8) or ceil(len / 4) (packed2)
   int chunks;            // ceil(len / 64): an item covers 64 positions
   int64_t items;         // G * chunks
-  bool vec_ok;           // 16-byte aligned rows
+  bool vec_ok;           // rows 16-byte aligned for the vector loads
+  bool packed2;          // 4 bases per byte (bpbc_sw_score_batch_packed2)
 };
 
 // 32 code bytes of one lane's pair at positions [c0, c0+32) (zeros past the
@@ -76,17 +83,32 @@ __device__ __forceinline__ void load32(const PackJob& J, int64_t pair, int64_t n
   }
 }
 
-// Fold, transpose across the warp and store one 32-position chunk.
-__device__ __forceinline__ void transpose_store(uint32_t (&w)[8], const uint32_t (&keep)[5],
-                                                const uint32_t (&rot)[5], uint2* dst, bool ok,
-                                                uint32_t& bad) {
-  bad |= (w[0] | w[1] | w[2] | w[3] | w[4] | w[5] | w[6] | w[7]) & 0xFCFCFCFCu;
+// 2-bit packed bases of one lane's pair, positions [c0, c0+64): 4 words, 16
+// bases each (bits past the row end are never stored).
+__device__ __forceinline__ void load64_packed2(const PackJob& J, int64_t pair, int64_t num_pairs,
+                                               int c0, uint32_t (&w)[4]) {
+  const uint8_t* row = J.codes + pair * J.stride + c0 / 4;
+  if (pair < num_pairs && J.vec_ok && c0 + 64 <= J.len) {
+    const uint4 a = __ldcs(reinterpret_cast<const uint4*>(row));
+    w[0] = a.x; w[1] = a.y; w[2] = a.z; w[3] = a.w;
+  } else {
 #pragma unroll
-  for (int q = 0; q < 8; ++q) w[q] &= 0x03030303u;
-  const uint32_t t = mad_lo(w[3], 64u, mad_lo(w[2], 16u, mad_lo(w[1], 4u, w[0])));
-  const uint32_t u = mad_lo(w[7], 64u, mad_lo(w[6], 16u, mad_lo(w[5], 4u, w[4])));
-  uint32_t H = (t & 0xAAAAAAAAu) | ((u >> 1) & 0x55555555u);
-  uint32_t L = ((t << 1) & 0xAAAAAAAAu) | (u & 0x55555555u);
+    for (int q = 0; q < 4; ++q) {
+      uint32_t v = 0;
+#pragma unroll
+      for (int bb = 0; bb < 4; ++bb) {
+        const int pos = c0 + 16 * q + 4 * bb;
+        if (pair < num_pairs && pos < J.len) v |= uint32_t(row[4 * q + bb]) << (8 * bb);
+      }
+      w[q] = v;
+    }
+  }
+}
+
+// Transpose the (H, L) words of one 32-position chunk across the warp and
+// store lane p's result at dst (position set by the caller's bit order).
+__device__ __forceinline__ void butterfly_store(uint32_t H, uint32_t L, const uint32_t (&keep)[5],
+                                                const uint32_t (&rot)[5], uint2* dst, bool ok) {
   // 32x32 bit transpose across the warp: stage j swaps the off-diagonal
   // j x j blocks between lanes l and l^j.  Lane l keeps its bits where
   // keep = 1 and takes the partner's word rotated by j into the others.
@@ -100,6 +122,21 @@ __device__ __forceinline__ void transpose_store(uint32_t (&w)[8], const uint32_t
   }
   if (ok) *dst = make_uint2(H, L);
 }
+
+// Fold, transpose across the warp and store one 32-position chunk.
+__device__ __forceinline__ void transpose_store(uint32_t (&w)[8], const uint32_t (&keep)[5],
+                                                const uint32_t (&rot)[5], uint2* dst, bool ok,
+                                                uint32_t& bad) {
+  bad |= (w[0] | w[1] | w[2] | w[3] | w[4] | w[5] | w[6] | w[7]) & 0xFCFCFCFCu;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) w[q] &= 0x03030303u;
+  const uint32_t t = mad_lo(w[3], 64u, mad_lo(w[2], 16u, mad_lo(w[1], 4u, w[0])));
+  const uint32_t u = mad_lo(w[7], 64u, mad_lo(w[6], 16u, mad_lo(w[5], 4u, w[4])));
+  uint32_t H = (t & 0xAAAAAAAAu) | ((u >> 1) & 0x55555555u);
+  uint32_t L = ((t << 1) & 0xAAAAAAAAu) | (u & 0x55555555u);
+  butterfly_store(H, L, keep, rot, dst, ok);
+}
+
 
 __global__ void __launch_bounds__(256) pack_kernel(const PackJob j0, const PackJob j1,
                                                    int64_t num_pairs,
@@ -128,12 +165,27 @@ __global__ void __launch_bounds__(256) pack_kernel(const PackJob j0, const PackJ
     const int64_t g = gq;
     const int c0 = int(li - gq * uint32_t(J.chunks)) * 64;
     const int64_t pair = g * 32 + lane;
+    uint2* row = J.planes + g * J.len;
+    if (J.packed2) {  // warp-uniform: 16 bytes per lane cover 64 positions
+      uint32_t w[4];
+      load64_packed2(J, pair, num_pairs, c0, w);
+      const int p2 = pos_of_bit_packed2(lane);
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        if (c0 + 32 * h < J.len) {  // warp-uniform
+          const uint32_t A = w[2 * h], B = w[2 * h + 1];
+          const uint32_t H = (A & 0xAAAAAAAAu) | ((B >> 1) & 0x55555555u);
+          const uint32_t L = ((A << 1) & 0xAAAAAAAAu) | (B & 0x55555555u);
+          butterfly_store(H, L, keep, rot, row + c0 + 32 * h + p2, c0 + 32 * h + p2 < J.len);
+        }
+      }
+      continue;
+    }
     // both 32-position halves are loaded before either is used (64 B per
     // lane in flight)
     uint32_t w0[8], w1[8];
     load32(J, pair, num_pairs, c0, w0);
     load32(J, pair, num_pairs, c0 + 32, w1);
-    uint2* row = J.planes + g * J.len;
     transpose_store(w0, keep, rot, row + c0 + mypos, c0 + mypos < J.len, bad);
     if (c0 + 32 < J.len)  // warp-uniform
       transpose_store(w1, keep, rot, row + c0 + 32 + mypos, c0 + 32 + mypos < J.len, bad);
@@ -141,14 +193,16 @@ __global__ void __launch_bounds__(256) pack_kernel(const PackJob j0, const PackJ
   if (__any_sync(0xFFFFFFFFu, bad != 0) && lane == 0) atomicOr(flags, BPBC_FLAG_BAD_BASE);
 }
 
-PackJob make_job(const uint8_t* codes, int64_t num_pairs, int len, uint2* planes) {
+PackJob make_job(const uint8_t* codes, int64_t num_pairs, int len, uint2* planes, bool packed2) {
   PackJob J;
   J.codes = codes;
   J.planes = planes;
   J.len = len > 0 ? len : 1;
+  J.packed2 = packed2;
+  J.stride = packed2 ? (J.len + 3) / 4 : J.len;
   J.chunks = (J.len + 63) / 64;
   J.items = (codes && len > 0) ? (num_pairs + 31) / 32 * J.chunks : 0;
-  J.vec_ok = (len % 16 == 0) && ((reinterpret_cast<uintptr_t>(codes) & 15) == 0);
+  J.vec_ok = (J.stride % 16 == 0) && ((reinterpret_cast<uintptr_t>(codes) & 15) == 0);
   return J;
 }
 
@@ -156,10 +210,10 @@ PackJob make_job(const uint8_t* codes, int64_t num_pairs, int len, uint2* planes
 
 cudaError_t launch_pack2(const uint8_t* codes_a, int len_a, uint2* planes_a,
                          const uint8_t* codes_b, int len_b, uint2* planes_b, int64_t num_pairs,
-                         uint32_t* flags, int num_sms, cudaStream_t stream) {
+                         uint32_t* flags, int num_sms, cudaStream_t stream, bool packed2) {
   if (num_pairs <= 0) return cudaSuccess;
-  const PackJob a = make_job(codes_a, num_pairs, len_a, planes_a);
-  const PackJob b = make_job(codes_b, num_pairs, len_b, planes_b);
+  const PackJob a = make_job(codes_a, num_pairs, len_a, planes_a, packed2);
+  const PackJob b = make_job(codes_b, num_pairs, len_b, planes_b, packed2);
   const int64_t items = a.items + b.items;
   if (items == 0) return cudaSuccess;
   if (a.items >= (int64_t(1) << 31) || b.items >= (int64_t(1) << 31)) return cudaErrorInvalidValue;
@@ -174,7 +228,8 @@ cudaError_t launch_pack2(const uint8_t* codes_a, int len_a, uint2* planes_a,
 cudaError_t launch_pack(const uint8_t* codes, int64_t num_pairs, int len, uint2* planes,
                         uint32_t* flags, int num_sms, cudaStream_t stream) {
   if (num_pairs <= 0 || len <= 0) return cudaSuccess;
-  return launch_pack2(codes, len, planes, nullptr, 0, nullptr, num_pairs, flags, num_sms, stream);
+  return launch_pack2(codes, len, planes, nullptr, 0, nullptr, num_pairs, flags, num_sms, stream,
+                      false);
 }
 
 }  // namespace bpbc

@@ -30,6 +30,9 @@
 #ifndef BPBC_S
 #error "compile with -DBPBC_S=<score width>"
 #endif
+#ifndef BPBC_MODE
+#error "compile with -DBPBC_MODE=<0 running max | 1 threshold flag>"
+#endif
 
 namespace bpbc {
 namespace {
@@ -44,6 +47,16 @@ __device__ __forceinline__ uint32_t mul_lo(uint32_t a, uint32_t b) {
   asm("mul.lo.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
   return r;
 }
+
+// Asynchronous 8-byte global -> shared copies (cp.async, no register
+// staging): the next group's query planes are fetched while the current
+// group runs, and read back with a short-latency LDS at the group switch.
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
+  const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
 template <int S, int R, int L, int CIRC, bool PAD, class K>
 __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const K k) {
@@ -81,41 +94,52 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
 #pragma unroll
     for (int r = 0; r < R; ++r) H[r][i] = 0;
   }
-  uint32_t xh[R], xl[R], nxh[R], nxl[R];
-  {
-    const uint2* xp = a.Xp + (gb < a.G ? gb : a.G - 1) * a.m + sl * R;
+  // my query planes: registers for the current group, a 2-slot shared ring
+  // for the current and the next group (slot = group index & 1)
+  __shared__ uint2 xring[4][2][32][R];  // [warp in block][slot][lane][row]
+  uint2 (*ring)[32][R] = xring[threadIdx.x >> 5];
+  uint32_t xh[R], xl[R];
+  auto fetch_x = [&](int64_t gidx, int slot) {  // gidx: group index in the stream
+    int64_t g = gb + gidx;
+    g = g < a.G ? g : a.G - 1;
+    const uint2* xp = a.Xp + g * a.m + sl * R;
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
-      const uint2 v = __ldg(xp + r);
-      nxh[r] = v.x;
-      nxl[r] = v.y;
-      xh[r] = xl[r] = 0;
-    }
-  }
+    for (int r = 0; r < R; ++r) cp_async8(&ring[slot][lane][r], xp + r);
+    cp_async_commit();
+  };
+  fetch_x(0, 0);
+#pragma unroll
+  for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
   const uint2* yp = a.Yp + gb * a.n - sl;
-  uint2 ynext = __ldg(yp);
   int cnt = sl;      // steps until my next group starts (J % n == 0)
   int64_t gi = -1;   // my current group within the stream
+  uint32_t flag = 0; // threshold mode: pairs with a cell > tau so far
 
-  for (int64_t tau = 0; tau < a.steps; ++tau) {
+  // One wavefront step with target planes y of my current column.
+  auto step = [&](const uint2 y) {
     uint32_t up[S];
 #pragma unroll
     for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
 
     if (cnt == 0) {  // column 0 of my next group (divergent, once per group)
       if (gi >= 0 && gi < Gs) {
-        uint32_t* dst = a.Mpart + ((gb + gi) * L + sl) * S;
-        if constexpr (CIRC == kExact) {
-          uint32_t F[S];
-          finish_exact<S, K::g>(M, F);  // M tracked D' = diag + w + g
-#pragma unroll
-          for (int i = 0; i < S; ++i) dst[i] = F[i];
+        if constexpr (BPBC_MODE == kModeThreshold) {
+          a.Mpart[(gb + gi) * L + sl] = flag;  // one flag word per lane
         } else {
+          uint32_t* dst = a.Mpart + ((gb + gi) * L + sl) * S;
+          if constexpr (CIRC == kExact) {
+            uint32_t F[S];
+            finish_exact<S, K::g>(M, F);  // M tracked D' = diag + w + g
 #pragma unroll
-          for (int i = 0; i < S; ++i) dst[i] = M[i];
+            for (int i = 0; i < S; ++i) dst[i] = F[i];
+          } else {
+#pragma unroll
+            for (int i = 0; i < S; ++i) dst[i] = M[i];
+          }
         }
       }
       ++gi;
+      flag = 0;
 #pragma unroll
       for (int i = 0; i < S; ++i) {
         M[i] = 0;
@@ -123,23 +147,18 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
 #pragma unroll
         for (int r = 0; r < R; ++r) H[r][i] = 0;
       }
-      int64_t nxt = gb + gi + 1;
-      nxt = nxt < a.G ? nxt : a.G - 1;
-      const uint2* xp = a.Xp + nxt * a.m + sl * R;
+      cp_async_wait_all();  // my own copies of group gi (issued n steps ago)
 #pragma unroll
       for (int r = 0; r < R; ++r) {
-        xh[r] = nxh[r];
-        xl[r] = nxl[r];
-        const uint2 v = __ldg(xp + r);
-        nxh[r] = v.x;
-        nxl[r] = v.y;
+        const uint2 v = ring[gi & 1][lane][r];
+        xh[r] = v.x;
+        xl[r] = v.y;
       }
+      fetch_x(gi + 1, int((gi + 1) & 1));  // slot of group gi - 1, no longer read
       cnt = a.n;
     }
     --cnt;
 
-    const uint2 y = ynext;
-    ynext = __ldg(yp + tau + 1);  // prefetch one step ahead (pads cover it)
     uint32_t dg[S], u[S];
 #pragma unroll
     for (int i = 0; i < S; ++i) {
@@ -156,7 +175,11 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
       } else {
         cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
       }
-      runmax<S, PAD>(M, dn, kill[r]);
+      if constexpr (BPBC_MODE == kModeThreshold) {
+        flag_gt<S, PAD>(flag, dn, a.tmask, kill[r]);
+      } else {
+        runmax<S, PAD>(M, dn, kill[r]);
+      }
 #pragma unroll
       for (int i = 0; i < S; ++i) {
         dg[i] = H[r][i];
@@ -166,6 +189,18 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     }
 #pragma unroll
     for (int i = 0; i < S; ++i) dtop[i] = up[i];
+  };
+
+  // Two steps per iteration with two target registers: each load lands in
+  // its own register half an iteration before use, so no register move
+  // waits on it (steps is rounded up to even; the pads cover the extra
+  // column and an extra step past the last group stores nothing).
+  uint2 y0 = __ldg(yp), y1;
+  for (int64_t tau = 0; tau < a.steps; tau += 2) {
+    y1 = __ldg(yp + tau + 1);
+    step(y0);
+    y0 = __ldg(yp + tau + 2);
+    step(y1);
   }
 }
 
@@ -187,9 +222,9 @@ __device__ __forceinline__ uint32_t mad_lo(uint32_t a, uint32_t b, uint32_t c) {
 // reads a zero row instead (border d[-1][j] = 0).  The partial
 // maxima go to Mpart[g][k][lane] (the extract kernel reduces stripes x lanes).
 // Everything else is the short kernel (same circuits, same wavefront).
-template <int S, int CIRC, class K>
+template <int S, int CIRC, class K, int R>
 __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a, const K k) {
-  constexpr int R = kStripeR, L = 32, LR = L * R;
+  constexpr int L = 32, LR = L * R;
   constexpr int SP = (S + 3) / 4 * 4;  // boundary words per column (uint4 aligned)
   const int sl = threadIdx.x & 31;
   const int64_t warp = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
@@ -215,20 +250,20 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
   }
 #pragma unroll
   for (int r = 0; r < R; ++r) kill[r] = 0;
-  uint32_t xh[R], xl[R], nxh[R], nxl[R];
-  auto load_x = [&](int64_t u) {  // query planes of unit u (clamped)
+  uint32_t xh[R], xl[R];
+  __shared__ uint2 xring[4][2][32][R];  // next unit's query planes (cp.async)
+  uint2 (*ring)[32][R] = xring[threadIdx.x >> 5];
+  auto fetch_x = [&](int64_t u) {  // query planes of unit u (clamped) -> slot u & 1
+    const int slot = int(u & 1);
     u = u < units ? u : units - 1;
     const int64_t g = gb + u / stripes;
     const int kk = int(u % stripes);
     const uint2* xp = a.Xp + g * a.m + kk * LR + sl * R;
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
-      const uint2 v = __ldg(xp + r);
-      nxh[r] = v.x;
-      nxl[r] = v.y;
-    }
+    for (int r = 0; r < R; ++r) cp_async8(&ring[slot][sl][r], xp + r);
+    cp_async_commit();
   };
-  load_x(0);
+  fetch_x(0);
 #pragma unroll
   for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
   const uint2* ycol = a.Yp;  // my current target column (valid dummy before unit 0)
@@ -239,6 +274,7 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
   bool store_bnd = false;       // last lane, not the last stripe
   int cnt = sl;
   int64_t vi = -1;
+  uint32_t flag = 0;  // threshold mode
 
   for (int64_t tau = 0; tau < a.steps; ++tau) {
     uint32_t up[S];
@@ -250,18 +286,23 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
       if (vi >= 0 && vi < units) {
         const int64_t g = gb + vi / stripes;
         const int kk = int(vi % stripes);
-        uint32_t* dst = a.Mpart + ((g * stripes + kk) * L + sl) * S;
-        if constexpr (CIRC == kExact) {
-          uint32_t F[S];
-          finish_exact<S, K::g>(M, F);
-#pragma unroll
-          for (int i = 0; i < S; ++i) dst[i] = F[i];
+        if constexpr (BPBC_MODE == kModeThreshold) {
+          a.Mpart[(g * stripes + kk) * L + sl] = flag;
         } else {
+          uint32_t* dst = a.Mpart + ((g * stripes + kk) * L + sl) * S;
+          if constexpr (CIRC == kExact) {
+            uint32_t F[S];
+            finish_exact<S, K::g>(M, F);
 #pragma unroll
-          for (int i = 0; i < S; ++i) dst[i] = M[i];
+            for (int i = 0; i < S; ++i) dst[i] = F[i];
+          } else {
+#pragma unroll
+            for (int i = 0; i < S; ++i) dst[i] = M[i];
+          }
         }
       }
       ++vi;
+      flag = 0;
       const int64_t uc = vi < units ? vi : units - 1;
       const int64_t g = gb + uc / stripes;
       const int kk = int(uc % stripes);
@@ -272,13 +313,15 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
 #pragma unroll
         for (int r = 0; r < R; ++r) H[r][i] = 0;
       }
+      cp_async_wait_all();
 #pragma unroll
       for (int r = 0; r < R; ++r) {
-        xh[r] = nxh[r];
-        xl[r] = nxl[r];
+        const uint2 v = ring[vi & 1][sl][r];
+        xh[r] = v.x;
+        xl[r] = v.y;
         kill[r] = (kk * LR + sl * R + r >= a.m) ? 0xFFFFFFFFu : 0u;
       }
-      load_x(vi + 1);
+      fetch_x(vi + 1);
       ycol = a.Yp + g * a.n;
       y = yfirst;
       {
@@ -330,7 +373,11 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
       } else {
         cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
       }
-      runmax<S, true>(M, dn, kill[r]);
+      if constexpr (BPBC_MODE == kModeThreshold) {
+        flag_gt<S, true>(flag, dn, a.tmask, kill[r]);
+      } else {
+        runmax<S, true>(M, dn, kill[r]);
+      }
 #pragma unroll
       for (int i = 0; i < S; ++i) {
         dg[i] = H[r][i];
@@ -365,13 +412,25 @@ void launch_sweep(const SweepArgs& a, const KRun& kr, int grid, int block, cudaS
   }
 }
 
-template <int S, int CIRC, class K>
+template <int S, int CIRC, class K, int R>
 void launch_striped(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
   if constexpr (K::kFixed) {
-    sw_sweep_striped_kernel<S, CIRC, K><<<grid, block, 0, st>>>(a, K{});
+    sw_sweep_striped_kernel<S, CIRC, K, R><<<grid, block, 0, st>>>(a, K{});
   } else {
-    sw_sweep_striped_kernel<S, CIRC, KRun><<<grid, block, 0, st>>>(a, kr);
+    sw_sweep_striped_kernel<S, CIRC, KRun, R><<<grid, block, 0, st>>>(a, kr);
   }
+}
+
+template <int S, int RV>
+void reg_striped(SweepEntry (*stab)[3][13]) {
+  constexpr int R = kStripeRV[RV];
+  using K211 = KFix<2, 1, 1>;
+  stab[RV][0][S - 4] = {&launch_striped<S, kExact, K211, R>,
+                        (const void*)&sw_sweep_striped_kernel<S, kExact, K211, R>};
+  stab[RV][1][S - 4] = {&launch_striped<S, kSat, K211, R>,
+                        (const void*)&sw_sweep_striped_kernel<S, kSat, K211, R>};
+  stab[RV][2][S - 4] = {&launch_striped<S, kSat, KRun, R>,
+                        (const void*)&sw_sweep_striped_kernel<S, kSat, KRun, R>};
 }
 
 template <int S, int RL, bool PAD>
@@ -393,18 +452,8 @@ void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
 
 #define BPBC_CAT2(a, b) a##b
 #define BPBC_CAT(a, b) BPBC_CAT2(a, b)
-void BPBC_CAT(register_striped_s, BPBC_S)(SweepEntry (*tab)[13]) {
-  using K211 = KFix<2, 1, 1>;
-  tab[0][BPBC_S - 4] = {
-      &launch_striped<BPBC_S, kExact, K211>,
-      (const void*)&sw_sweep_striped_kernel<BPBC_S, kExact, K211>};
-  tab[1][BPBC_S - 4] = {&launch_striped<BPBC_S, kSat, K211>,
-                        (const void*)&sw_sweep_striped_kernel<BPBC_S, kSat, K211>};
-  tab[2][BPBC_S - 4] = {&launch_striped<BPBC_S, kSat, KRun>,
-                        (const void*)&sw_sweep_striped_kernel<BPBC_S, kSat, KRun>};
-}
-
-void BPBC_CAT(register_sweep_s, BPBC_S)(SweepEntry (*tab)[kNumRL][13]) {
+#define BPBC_REGNAME BPBC_CAT(BPBC_CAT(BPBC_CAT(register_sweep_s, BPBC_S), _m), BPBC_MODE)
+void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13]) {
   reg_rl<BPBC_S, 0, false>(tab);
   reg_rl<BPBC_S, 1, false>(tab);
   reg_rl<BPBC_S, 2, false>(tab);
@@ -413,6 +462,8 @@ void BPBC_CAT(register_sweep_s, BPBC_S)(SweepEntry (*tab)[kNumRL][13]) {
   reg_rl<BPBC_S, 1, true>(tab);
   reg_rl<BPBC_S, 2, true>(tab);
   reg_rl<BPBC_S, 3, true>(tab);
+  reg_striped<BPBC_S, 0>(stab);
+  reg_striped<BPBC_S, 1>(stab);
 }
 
 }  // namespace bpbc

@@ -114,3 +114,24 @@ def encode(s: str) -> np.ndarray:
     """'ATGC' string -> codes (A=0, T=1, G=2, C=3; P:L51)."""
     table = {"A": 0, "T": 1, "G": 2, "C": 3}
     return np.array([table[c] for c in s.upper()], dtype=np.uint8)
+
+
+def pack2bit(codes: np.ndarray) -> np.ndarray:
+    """Input-format helper (no method arithmetic): uint8 codes [P, len] ->
+    2-bit packed rows [P, ceil(len/4)], base i in bits 2(i%4) of byte i//4
+    (the layout of bpbc_sw_score_batch_packed2, include/bpbc_sw.h)."""
+    codes = np.asarray(codes, dtype=np.uint8)
+    P, ln = codes.shape
+    w = (ln + 3) // 4
+    pad = np.zeros((P, 4 * w), dtype=np.uint8)
+    pad[:, :ln] = codes & 3
+    q = pad.reshape(P, w, 4)
+    return np.ascontiguousarray(q[:, :, 0] | (q[:, :, 1] << 2) | (q[:, :, 2] << 4) | (q[:, :, 3] << 6))
+
+
+def unpack2bit(packed: np.ndarray, ln: int) -> np.ndarray:
+    """Inverse of pack2bit."""
+    packed = np.asarray(packed, dtype=np.uint8)
+    P = packed.shape[0]
+    out = np.stack([(packed >> (2 * k)) & 3 for k in range(4)], axis=2).reshape(P, -1)
+    return np.ascontiguousarray(out[:, :ln])

@@ -291,3 +291,83 @@ def test_m256_wide_width_uses_stripes(s):
     q, t = synth.gen_pairs(777 + s, 200, 200, 240, planted=True)
     check_full(q, t, 31, -1, -1, s=s)
     assert bpbc.last_plan(0)["rows_per_lane"] == 4
+
+
+# ---------------------------------------------------------------- 2-bit packed input (NEXT-1)
+
+
+@pytest.mark.parametrize("m,n", [(64, 64), (128, 128), (40, 56), (1, 9), (77, 300), (300, 520),
+                                 (256, 256)])
+def test_packed2_device_matches_oracle(m, n):
+    q, t = synth.gen_pairs(6060 + m + n, 999, m, n, planted=True)
+    q2 = torch.from_numpy(synth.pack2bit(q)).to(DEV)
+    t2 = torch.from_numpy(synth.pack2bit(t)).to(DEV)
+    got = bpbc.score_batch_packed2(q2, t2, m, n, 2, -1, -1).cpu().numpy()
+    s = bpbc.default_score_bits(2, m, n)
+    np.testing.assert_array_equal(got, oracle.sw_batch(q, t, 2, -1, -1, score_bits=s))
+
+
+def test_packed2_host_matches_u8_path():
+    q, t = synth.gen_pairs(7070, 70000, 128, 128, planted=True)  # several host chunks
+    got = bpbc.score_batch_host_packed2(synth.pack2bit(q), synth.pack2bit(t), 128, 128, 2, -1, -1, 9)
+    ref = bpbc.score_batch_host(q, t, 2, -1, -1, 9)
+    np.testing.assert_array_equal(got, ref)
+    idx = np.arange(0, 70000, 97)
+    np.testing.assert_array_equal(got[idx], oracle.sw_batch(q[idx], t[idx], 2, -1, -1, score_bits=9))
+
+
+# ---------------------------------------------------------------- threshold filter (NEXT-2)
+
+
+def _check_filter(q, t, tau, match=2, mismatch=-1, gap=-1, s=None):
+    m, n = q.shape[1], t.shape[1]
+    if s is None:
+        s = bpbc.default_score_bits(match, m, n)
+    dq = torch.from_numpy(np.ascontiguousarray(q)).to(DEV)
+    dt = torch.from_numpy(np.ascontiguousarray(t)).to(DEV)
+    mask, count, idx = bpbc.filter_batch(dq, dt, tau, match, mismatch, gap, score_bits=s)
+    P = q.shape[0]
+    exact = oracle.sw_batch(q, t, match, mismatch, gap)  # uncapped scores
+    want = np.nonzero(exact > tau)[0]
+    words = mask.cpu().numpy().view(np.uint32)
+    bits = ((words[:, None] >> np.arange(32, dtype=np.uint32)[None, :]) & 1).reshape(-1)[:P]
+    np.testing.assert_array_equal(np.nonzero(bits)[0], want)
+    assert (((words[:, None] >> np.arange(32, dtype=np.uint32)[None, :]) & 1).reshape(-1)[P:] == 0).all()
+    c = int(count.item())
+    assert c == want.size
+    np.testing.assert_array_equal(idx.cpu().numpy()[:c], want)
+    return want.size
+
+
+@pytest.mark.parametrize("tau", [0, 1, 20, 45, 60, 100, 127])
+def test_filter_c1_thresholds(tau):
+    q, t = synth.gen_pairs(synth.seed_for_config(1), 1024, 64, 64, planted=True)
+    _check_filter(q, t, tau, s=8)
+
+
+@pytest.mark.parametrize("P,m,n,tau", [(1000, 40, 56, 30), (33, 128, 128, 100), (4096, 128, 128, 110),
+                                       (300, 300, 300, 200), (257, 64, 1024, 70), (100, 9, 1, 1)])
+def test_filter_shapes(P, m, n, tau):
+    q, t = synth.gen_pairs(8080 + m + n, P, m, n, planted=True)
+    _check_filter(q, t, tau)
+
+
+@pytest.mark.parametrize("consts", [(1, -1, -1), (3, -2, -1), (1, 0, 0), (5, -3, -4)])
+def test_filter_runtime_constants(consts):
+    q, t = synth.gen_pairs(8181, 500, 37, 61, planted=True)
+    c1, mm, g = consts
+    for tau in (5, 20, 40):
+        _check_filter(q, t, tau, c1, mm, g, 12)
+
+
+def test_filter_threshold_edges():
+    q, t = synth.gen_pairs(8282, 70, 20, 30, planted=True)
+    assert _check_filter(q, t, 40) == 0  # >= match * min(m, n): nothing can exceed it
+    dq = torch.from_numpy(q).to(DEV)
+    dt = torch.from_numpy(t).to(DEV)
+    with pytest.raises(bpbc.BPBCError) as ei:
+        bpbc.filter_batch(dq, dt, 255, score_bits=8)  # > 2^s - 2
+    assert ei.value.status == _lib.BPBC_ERR_INVALID_ARG
+    with pytest.raises(bpbc.BPBCError) as ei:
+        bpbc.filter_batch(dq, dt, -1, score_bits=8)
+    assert ei.value.status == _lib.BPBC_ERR_INVALID_ARG

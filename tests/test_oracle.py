@@ -285,3 +285,16 @@ def test_generator_c_matches_numpy_definition():
     q, _ = synth.gen_pairs(1, 4096, 64, 1)
     frac = np.bincount(q.ravel(), minlength=4) / q.size
     assert np.all(np.abs(frac - 0.25) < 0.01)
+
+
+def test_pack2bit_roundtrip_and_layout():
+    """Input-format helper of the packed2 entry points: base i in bits 2(i%4)
+    of byte i//4 (include/bpbc_sw.h), lossless for codes 0..3."""
+    rng = np.random.default_rng(5)
+    for ln in (1, 3, 4, 5, 31, 64, 129):
+        c = rng.integers(0, 4, size=(7, ln), dtype=np.uint8)
+        p = synth.pack2bit(c)
+        assert p.shape == (7, (ln + 3) // 4)
+        np.testing.assert_array_equal(synth.unpack2bit(p, ln), c)
+    # hand example: ATGC -> 0 | 1<<2 | 2<<4 | 3<<6 = 0b11100100
+    assert synth.pack2bit(synth.encode("ATGC")[None, :])[0, 0] == 0b11100100
