@@ -322,6 +322,38 @@ def main():
                         "ascending indices (P:L231)"}
         del fmask, fidx, fcnt
 
+    # ---------------- wordwise comparator (NEXT-4) on the same resident batch
+    wordwise = None
+    if not args.no_filter and min(m, n) <= 256:
+        wws = torch.empty(max(ws.numel(), 1), dtype=torch.uint8, device=dev)
+        wout = torch.empty(P, dtype=torch.int32, device=dev)
+
+        def wstep():
+            bpbc.score_batch_wordwise(dq, dt, *CONSTS, out=wout)
+
+        for _ in range(args.warmup):
+            wstep()
+        wk = max(3, min(args.steps, 10))
+        ws0 = [torch.cuda.Event(enable_timing=True) for _ in range(wk)]
+        ws1 = [torch.cuda.Event(enable_timing=True) for _ in range(wk)]
+        torch.cuda.synchronize()
+        for k in range(wk):
+            flush.zero_()
+            ws0[k].record()
+            wstep()
+            ws1[k].record()
+        torch.cuda.synchronize()
+        w_ms = sum(x.elapsed_time(y) for x, y in zip(ws0, ws1))
+        wv = P * m * n * wk / (w_ms / 1e3) / 1e9
+        cap = (1 << s) - 1
+        agree = bool(torch.equal(torch.clamp(wout, max=cap), out))
+        wordwise = {"value": round(wv, 2), "unit": "GCUPS", "ms_per_step": round(w_ms / wk, 4),
+                    "bitwise_over_wordwise": round(gcups / world / wv, 3) if wv else None,
+                    "agrees_with_bitwise": agree,
+                    "what": "bpbc_sw_score_batch_wordwise: ordinary-integer DP, 16-bit SIMD, "
+                            "2 pairs per warp register (the paper's GPU wordwise row, P:L407)"}
+        del wws, wout
+
     # ---------------- end to end through the host-buffer C call
     e2e = e2e_packed2 = None
     if not args.no_e2e:
@@ -436,7 +468,7 @@ def main():
                        "m": m, "n": n, "score_bits": s, "parallelism": f"dp{world} (pair shards)",
                        "l2": "inputs 320 MiB > 126 MB L2, plus a 256 MiB L2 flush between steps",
                        "plan": plan},
-            "e2e": e2e, "e2e_packed2": e2e_packed2, "filter": filt, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,
+            "e2e": e2e, "e2e_packed2": e2e_packed2, "filter": filt, "wordwise": wordwise, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,
             # ours per step and rank: pack (query+target), sweep, extract
             "gpu_launches": 3 * args.steps * world, "parity": parity}
     print(json.dumps(line), flush=True)

@@ -182,6 +182,22 @@ int bpbc_sw_filter_batch(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8_t *
                          void *workspace, size_t workspace_bytes, void *stream);
 
 /*
+ * Wordwise comparator: the same scores computed WITHOUT
+ * the bitwise technique -- ordinary integer DP cells, the paper's "GPU
+ * wordwise" implementation (Table IV) written for sm_100a with
+ * 16-bit SIMD (two pairs per warp register) -- so the BPBC path's gain can be
+ * measured on the same GPU.  Returns the exact max local score (no width
+ * cap).  min(m, n) <= 256 and the scores must fit 16 bits (else
+ * UNSUPPORTED).  workspace: device, >= bpbc_sw_wordwise_workspace_bytes, or
+ * NULL for the ctx-owned buffer.  Asynchronous on `stream`.
+ */
+int bpbc_sw_wordwise_workspace_bytes(int64_t num_pairs, size_t *bytes);
+int bpbc_sw_score_batch_wordwise(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8_t *target,
+                                 int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                                 int32_t mismatch, int32_t gap, int32_t *out_scores,
+                                 void *workspace, size_t workspace_bytes, void *stream);
+
+/*
  * W2B step alone: bit-transpose base codes into planes.
  * codes   device, uint8 [num_pairs][len].
  * planes  device, uint32 [ceil(num_pairs/32)][len][2]: [g][i][0] = X^H_i,

@@ -44,6 +44,10 @@ SIGNATURES = {
     "bpbc_sw_filter_batch": (_c.c_int, [_vp, _vp, _vp, _c.c_int64, _c.c_int32, _c.c_int32,
                                         _c.c_int32, _c.c_int32, _c.c_int32, _c.c_int32,
                                         _c.c_int32, _vp, _vp, _vp, _vp, _c.c_size_t, _vp]),
+    "bpbc_sw_wordwise_workspace_bytes": (_c.c_int, [_c.c_int64, _c.POINTER(_c.c_size_t)]),
+    "bpbc_sw_score_batch_wordwise": (_c.c_int, [_vp, _vp, _vp, _c.c_int64, _c.c_int32,
+                                                _c.c_int32, _c.c_int32, _c.c_int32, _c.c_int32,
+                                                _vp, _vp, _c.c_size_t, _vp]),
     "bpbc_sw_pack": (_c.c_int, [_vp, _vp, _c.c_int64, _c.c_int32, _vp, _vp]),
     "bpbc_sw_untranspose": (_c.c_int, [_vp, _vp, _c.c_int64, _c.c_int32, _c.c_int32,
                                        _c.c_int64, _c.c_int32, _vp, _vp]),

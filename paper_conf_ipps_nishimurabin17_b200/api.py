@@ -145,6 +145,31 @@ def filter_batch(query: torch.Tensor, target: torch.Tensor, threshold: int, matc
     return mask, count, idx
 
 
+def score_batch_wordwise(query: torch.Tensor, target: torch.Tensor, match: int = 2,
+                         mismatch: int = -1, gap: int = -1, out: torch.Tensor | None = None,
+                         workspace: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """bpbc_sw_score_batch_wordwise: the wordwise (non-bitwise) 16-bit SIMD
+    comparator on the same inputs; exact int32 scores (no width cap)."""
+    if not (query.is_cuda and target.is_cuda):
+        raise ValueError("score_batch_wordwise needs CUDA tensors")
+    if query.dtype != torch.uint8 or target.dtype != torch.uint8:
+        raise TypeError("query/target must be uint8 base codes")
+    query, target = query.contiguous(), target.contiguous()
+    P, m = query.shape
+    n = target.shape[1]
+    dev = query.device.index if query.device.index is not None else torch.cuda.current_device()
+    if out is None:
+        out = torch.empty(P, dtype=torch.int32, device=query.device)
+    ws_ptr, ws_bytes = None, 0
+    if workspace is not None:
+        ws_ptr, ws_bytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
+    ctx = _ctx(dev)
+    check(_lib.load().bpbc_sw_score_batch_wordwise(
+        ctx, query.data_ptr(), target.data_ptr(), P, m, n, match, mismatch, gap, out.data_ptr(),
+        ws_ptr, ws_bytes, _stream_ptr(stream, query.device)), ctx)
+    return out
+
+
 def score_batch_packed2(query2: torch.Tensor, target2: torch.Tensor, m: int, n: int,
                         match: int = 2, mismatch: int = -1, gap: int = -1,
                         score_bits: int | None = None, out: torch.Tensor | None = None,

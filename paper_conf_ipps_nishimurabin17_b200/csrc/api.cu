@@ -55,14 +55,16 @@ namespace {
 
 SweepEntry g_table[2][kNumVariants][kNumRL][13];  // [mode][variant][rl][S - 4]
 SweepEntry g_striped[2][kNumStripeRV][3][13];     // [mode][stripe R][kind][S - 4]
+SweepEntry g_mw[2][kNumMw][3][13];                // [mode][(R, W)][kind][S - 4]
 std::once_flag g_table_once;
 
 void init_table() {
   memset(g_table, 0, sizeof(g_table));
   memset(g_striped, 0, sizeof(g_striped));
+  memset(g_mw, 0, sizeof(g_mw));
 #define BPBC_REG(S)                                      \
-  register_sweep_s##S##_m0(g_table[0], g_striped[0]); \
-  register_sweep_s##S##_m1(g_table[1], g_striped[1]);
+  register_sweep_s##S##_m0(g_table[0], g_striped[0], g_mw[0]); \
+  register_sweep_s##S##_m1(g_table[1], g_striped[1], g_mw[1]);
   BPBC_REG(4)
   BPBC_REG(5)
   BPBC_REG(6)
@@ -108,7 +110,8 @@ Layout layout(int64_t P, int mq, int nt) {
   Layout L;
   L.G = (P + 31) / 32;
   // room for the striped kernel whenever the plan may pick it (m > 128)
-  L.stripes = mq > 128 ? (mq + kMinStripeRows - 1) / kMinStripeRows : 1;
+  // room for the striped / multi-warp kernels' partials: 32 lanes per 64 rows
+  L.stripes = (mq + kMinStripeRows - 1) / kMinStripeRows;
   const int64_t xbytes = (L.G * mq + kXBackPad) * 8;
   const int64_t ybytes = (kYFrontPad + L.G * nt + nt + kYBackPadExtra) * 8;
   const int64_t mpbytes = L.G * L.stripes * 32 * 16 * 4;
@@ -132,24 +135,15 @@ Layout layout(int64_t P, int mq, int nt) {
 
 struct Plan {
   int circuit, consts, rl, width, cap;
-  int stripe_rv = 1;  // striped kernels: index into kStripeRV
+  int stripe_rv = 0;  // striped kernels: index into kStripeRV
   bool pad;
   int ops;
 };
 
-// Rows per lane of the striped kernel: 4 unless BPBC_STRIPE_R=2 is set in the
-// environment (a tuning knob for benchmarks; read once).
-int stripe_rv_default() {
-  static const int rv = [] {
-    const char* v = getenv("BPBC_STRIPE_R");
-    return (v && atoi(v) == 2) ? 0 : 1;
-  }();
-  return rv;
-}
 
 // Choose the circuit, the evaluated width and the tiling.
 int make_plan(int mq, int c1, int c2, int g, int S, Plan* p) {
-  p->stripe_rv = stripe_rv_default();
+  p->stripe_rv = 0;
   if (mq <= 32) p->rl = 0;
   else if (mq <= 64) p->rl = 1;
   else if (mq <= 128) p->rl = 2;
@@ -211,9 +205,31 @@ struct Dispatch {
   Plan plan;
   SweepEntry ent;
   bool striped;
-  int R, L;
+  int mw = -1;          // multi-warp variant (index into kMwR / kMwW), -1 = none
+  int R, L, W = 1;      // rows per lane, lanes per group, warps per group
   int64_t cap_streams;  // resident streams (before the boundary-buffer cap)
 };
+
+// Multi-warp variant for this plan, or -1: long queries up to
+// 512 rows (R = 4, one warp per 128 rows) and the wide-plane 129..256 case.
+int pick_mw(int mq, const Plan& p, int64_t G, int64_t short_cap) {
+  auto idx = [](int R, int W) {
+    for (int i = 0; i < kNumMw; ++i)
+      if (kMwR[i] == R && kMwW[i] == W) return i;
+    return -1;
+  };
+  if (p.rl < 0) {  // the plan wants stripes
+    if (mq <= 512) return idx(4, (mq + 127) / 128 < 2 ? 2 : (mq + 127) / 128);
+    return -1;
+  }
+  // Few long groups (the paper's shape, G = 1024): splitting 128 rows over
+  // two R = 2 warps was measured 9 % SLOWER than one R = 4 warp per group
+  // (4 566 vs 5 016 GCUPS) -- the per-cell overhead of R = 2 outweighs the
+  // doubled warp count -- so the small-G split is only taken on request.
+  if (getenv("BPBC_SPLIT_FEW_GROUPS") && G > 0 && G * 2 <= short_cap && mq > 64 && mq <= 256)
+    return idx(2, (mq + 63) / 64 <= 2 ? 2 : 4);
+  return -1;
+}
 
 // Cap on resident sweep blocks per SM: BPBC_MAX_BLOCKS_PER_SM in the
 // environment (tuning knob for benchmarks; read once), else none.
@@ -242,7 +258,7 @@ int occupancy_blocks(const void* func) {  // cached per kernel
 }
 
 int make_dispatch(bpbc_sw_ctx* ctx, int mq, int c1, int c2, int g, int S, Dispatch* d,
-                  int mode = kModeMax) {
+                  int mode = kModeMax, int64_t G = 0) {
   int rc = make_plan(mq, c1, c2, g, S, &d->plan);
   if (rc != BPBC_OK) return rc;
   std::call_once(g_table_once, init_table);
@@ -261,6 +277,27 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int c1, int c2, int g, int S, Dispat
   if (nb < 0) return cuda_fail(ctx, cudaGetLastError(), "occupancy");
   if (max_blocks_env() > 0 && nb > max_blocks_env()) nb = max_blocks_env();
   d->cap_streams = int64_t(ctx->num_sms) * nb * 4 * (32 / d->L);
+  d->mw = getenv("BPBC_NO_MULTIWARP") ? -1 : pick_mw(mq, plan, G, d->cap_streams);
+  if (d->mw >= 0) {
+    const SweepEntry e =
+        g_mw[mode][d->mw][plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]
+            [plan.width - 4];
+    if (e.launch) {
+      d->ent = e;
+      d->striped = false;
+      d->R = kMwR[d->mw];
+      d->W = kMwW[d->mw];
+      d->L = 32;
+      int nbm = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nbm, e.func, 32 * d->W, 0) !=
+          cudaSuccess)
+        return cuda_fail(ctx, cudaGetLastError(), "occupancy");
+      if (nbm < 1) nbm = 1;
+      d->cap_streams = int64_t(ctx->num_sms) * nbm;  // one stream per block
+    } else {
+      d->mw = -1;
+    }
+  }
   return BPBC_OK;
 }
 
@@ -292,7 +329,7 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   }
   const int c1 = match, c2 = -mismatch, g = -gap;
   Dispatch dsp;
-  int rc = make_dispatch(ctx, mq, c1, c2, g, S, &dsp, o.mode);
+  int rc = make_dispatch(ctx, mq, c1, c2, g, S, &dsp, o.mode, (P + 31) / 32);
   if (rc != BPBC_OK) return rc;
   const Plan& plan = dsp.plan;
   const Layout lay = layout(P, mq, nt);
@@ -312,8 +349,9 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   if (ev[1]) cudaEventRecord(ev[1], st);
   const bool striped = dsp.striped;
   const SweepEntry ent = dsp.ent;
-  const int R = dsp.R, L = dsp.L;
-  const int64_t segs = 32 / L;
+  const int R = dsp.R, L = dsp.L, W = dsp.W;
+  const bool mw = dsp.mw >= 0;
+  const int64_t segs = mw ? 1 : 32 / L;
   int64_t cap_streams = dsp.cap_streams;
   if (striped && cap_streams > lay.bnd_streams) cap_streams = lay.bnd_streams;
   SweepArgs a;
@@ -329,7 +367,7 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   // [nb - 1, nb] minimising that (ties -> more warps for latency hiding);
   // the streams then split the groups as evenly as possible (base / rem).
   {
-    const int64_t per_block = 4 * segs;
+    const int64_t per_block = mw ? 1 : 4 * segs;
     const int64_t nb = cap_streams / (int64_t(ctx->num_sms) * per_block);
     int64_t best_b = nb > 0 ? nb : 1, best_t = -1;
     for (int64_t b = nb; b >= 1 && b >= nb - 1; --b) {
@@ -350,19 +388,22 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   a.bnd = reinterpret_cast<uint32_t*>(ws + lay.bnd_off);
   a.bzero = reinterpret_cast<const uint32_t*>(ws + lay.zero_off);
   a.steps = (a.base + (a.rem > 0 ? 1 : 0)) * a.stripes * int64_t(nt) + L;
+  if (mw) a.steps += int64_t(W - 1) * 64 + 31;  // warp lag (kMwLag), then whole phases
   a.steps += a.steps & 1;  // the short kernel runs two steps per iteration
+  if (mw) a.steps = (a.steps + 31) / 32 * 32;
   if (striped) {
     e = cudaMemsetAsync(ws + lay.zero_off, 0, 256, st);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "memset(zero row)");
   }
   const int64_t warps = (a.streams + segs - 1) / segs;
-  const int grid = int((warps + 3) / 4);
+  const int grid = mw ? int(a.streams) : int((warps + 3) / 4);
+  const int block = mw ? 32 * W : 128;
   KRun kr;
   memset(&kr, 0, sizeof(kr));
-  const int W = plan.width;
+  const int Wd = plan.width;
   for (int i = 0; i < 16; ++i) {
     kr.c1mask[i] = (c1 >> i) & 1 ? 0xFFFFFFFFu : 0u;
-    kr.nmask[i] = ((((1 << W) - c2) & ((1 << W) - 1)) >> i) & 1 ? 0xFFFFFFFFu : 0u;
+    kr.nmask[i] = ((((1 << Wd) - c2) & ((1 << Wd) - 1)) >> i) & 1 ? 0xFFFFFFFFu : 0u;
     kr.gmask[i] = (g >> i) & 1 ? 0xFFFFFFFFu : 0u;
   }
   kr.zmask = c2 == 0 ? 0xFFFFFFFFu : 0u;
@@ -370,24 +411,25 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   // circuit, whose D' carries the offset g)
   const int tcmp = o.threshold + (plan.circuit == kExact ? g : 0);
   for (int i = 0; i < 16; ++i) a.tmask[i] = (tcmp >> i) & 1 ? 0xFFFFFFFFu : 0u;
-  ent.launch(a, kr, grid, 128, st);
+  ent.launch(a, kr, grid, block, st);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(ctx, e, "sweep");
   if (ev[2]) cudaEventRecord(ev[2], st);
   if (o.mode == kModeThreshold) {
-    e = launch_filter_finish(Mpart, lay.G, L * a.stripes, P, o.mask, o.indices, o.count,
+    e = launch_filter_finish(Mpart, lay.G, L * a.stripes * W, P, o.mask, o.indices, o.count,
                              o.scratch, o.scratch_bytes, ctx->num_sms, st);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "filter epilogue");
   } else {
-    e = launch_extract(Mpart, lay.G, L * a.stripes, W, P, plan.cap, o.scores, ctx->num_sms, st);
+    e = launch_extract(Mpart, lay.G, L * a.stripes * W, plan.width, P, plan.cap, o.scores,
+                       ctx->num_sms, st);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "extract");
   }
   if (ev[3]) cudaEventRecord(ev[3], st);
 
   ctx->plan_circuit = plan.circuit;
-  ctx->plan_width = W;
+  ctx->plan_width = Wd;
   ctx->plan_R = R;
-  ctx->plan_L = L;
+  ctx->plan_L = L * W;  // lanes per group (over all its warps)
   ctx->plan_ops = plan.ops;
   ctx->plan_streams = a.streams;
   return BPBC_OK;
@@ -678,6 +720,42 @@ int bpbc_sw_filter_batch(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* 
   }
   return run_device(ctx, query, target, num_pairs, m, n, match, mismatch, gap, score_bits, o, ws,
                     st, false);
+}
+
+int bpbc_sw_wordwise_workspace_bytes(int64_t num_pairs, size_t* bytes) {
+  if (!bytes || num_pairs < 0) return BPBC_ERR_INVALID_ARG;
+  *bytes = wordwise_workspace_bytes(num_pairs);
+  return BPBC_OK;
+}
+
+int bpbc_sw_score_batch_wordwise(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target,
+                                 int64_t num_pairs, int32_t m, int32_t n, int32_t match,
+                                 int32_t mismatch, int32_t gap, int32_t* out_scores,
+                                 void* workspace, size_t workspace_bytes, void* stream) {
+  if (!ctx) return BPBC_ERR_INVALID_ARG;
+  int rc = validate_common(num_pairs, m, n, match, mismatch, gap, BPBC_MAX_SCORE_BITS);
+  if (rc != BPBC_OK) return rc;
+  const int mq = m < n ? m : n, nt = m < n ? n : m;
+  const int c2 = -mismatch, g = -gap, k0 = c2 > g ? c2 : g;
+  if (mq > 256) return BPBC_ERR_UNSUPPORTED;                       // R <= 8 rows per lane
+  if (int64_t(k0) + int64_t(match) * mq + match + c2 > 65535) return BPBC_ERR_UNSUPPORTED;
+  if (num_pairs == 0) return BPBC_OK;
+  if (!query || !target || !out_scores) return BPBC_ERR_INVALID_ARG;
+  DeviceGuard dg(ctx->device);
+  const size_t need = wordwise_workspace_bytes(num_pairs);
+  void* ws = workspace;
+  if (ws) {
+    if (workspace_bytes < need) return BPBC_ERR_INVALID_ARG;
+  } else {
+    rc = ensure_ws(ctx, need);
+    if (rc != BPBC_OK) return rc;
+    ws = ctx->ws;
+  }
+  const uint8_t* qx = m <= n ? query : target;  // the shorter sequence plays the rows (R17)
+  const uint8_t* ty = m <= n ? target : query;
+  cudaError_t e = launch_wordwise(qx, ty, num_pairs, mq, nt, match, c2, g, out_scores, ws,
+                                  ctx->num_sms, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? BPBC_OK : cuda_fail(ctx, e, "wordwise");
 }
 
 int bpbc_sw_score_batch_packed2(bpbc_sw_ctx* ctx, const uint8_t* query2, const uint8_t* target2,

@@ -12,9 +12,9 @@ namespace bpbc {
 // the Y stream of a warp is read at virtual column J = tau - lane, which runs
 // up to L columns before its first group and up to n + L columns past its
 // last.
-constexpr int64_t kYFrontPad = 64;   // uint2 words before Y plane 0
+constexpr int64_t kYFrontPad = 512;  // uint2 words before Y plane 0 (multi-warp lag)
 constexpr int64_t kXBackPad = 512;   // uint2 words after the last X group
-constexpr int64_t kYBackPadExtra = 128;
+constexpr int64_t kYBackPadExtra = 640;
 
 enum Circuit : int { kExact = 0, kSat = 1 };
 enum Mode : int { kModeMax = 0, kModeThreshold = 1 };  // running max / sticky flag
@@ -45,9 +45,13 @@ struct SweepArgs {
 };
 
 // Long queries: stripes of R rows per lane x 32 lanes, R in kStripeRV.
-constexpr int kNumStripeRV = 2;
-constexpr int kStripeRV[kNumStripeRV] = {2, 4};
+constexpr int kNumStripeRV = 1;
+constexpr int kStripeRV[kNumStripeRV] = {4};  // R = 2 measured 1.7x slower at C5
 constexpr int kMinStripeRows = 64;  // workspace is sized for the smallest stripes
+// Multi-warp groups (sw_sweep_mw_kernel): (R rows per lane, W warps per group)
+constexpr int kNumMw = 4;
+constexpr int kMwR[kNumMw] = {2, 2, 4, 4};
+constexpr int kMwW[kNumMw] = {2, 4, 2, 4};
 constexpr int kMaxShortRows = 256;     // m <= 256: the short kernel
 constexpr int64_t kMaxStripeStreams = 4096;
 constexpr int64_t kMaxBoundaryBytes = int64_t(1) << 30;
@@ -70,8 +74,10 @@ SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
 // short kernel, stab: [stripe R variant][striped kind][S-4] (0 exact (+2,-1,-1), 1 saturating
 // (+2,-1,-1), 2 saturating runtime constants).
 #define BPBC_DECLARE_REG(S)                                                       \
-  void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13]); \
-  void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13]);
+  void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13], \
+                                SweepEntry (*mtab)[3][13]);                               \
+  void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13], \
+                                SweepEntry (*mtab)[3][13]);
 BPBC_DECLARE_REG(4)
 BPBC_DECLARE_REG(5)
 BPBC_DECLARE_REG(6)
@@ -101,6 +107,11 @@ cudaError_t launch_filter_finish(const uint32_t* partial, int64_t num_groups, in
                                  int64_t num_pairs, uint32_t* mask, int64_t* indices,
                                  int64_t* count, void* scratch, size_t scratch_bytes,
                                  int num_sms, cudaStream_t stream);
+// wordwise.cu: the wordwise 16-bit SIMD comparator (NEXT-4)
+size_t wordwise_workspace_bytes(int64_t num_pairs);
+cudaError_t launch_wordwise(const uint8_t* q, const uint8_t* t, int64_t P, int mq, int nt,
+                            int c1, int c2, int g, int32_t* out, void* ws, int num_sms,
+                            cudaStream_t st);
 // extract.cu
 cudaError_t launch_extract(const uint32_t* partial, int64_t num_groups, int lanes, int s,
                            int64_t num_pairs, int32_t cap, int32_t* out, int num_sms,

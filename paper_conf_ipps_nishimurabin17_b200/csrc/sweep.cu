@@ -403,6 +403,210 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
   }
 }
 
+// ---------------------------------------------------------------------------
+// Multi-warp groups: the W warps of a block share one group stream and warp w
+// owns rows [w*32R, (w+1)*32R) of every group, running kMwLag steps behind
+// warp w-1 (lane l of warp w works on column J = tau - l - w*kMwLag).  The
+// bottom row of warp w (its lane 31) reaches lane 0 of warp w+1 through a
+// ring of kMwRing columns in shared memory; a __syncthreads every 32 steps
+// orders the writes before the reads: a column is read kMwLag - 31 = 33 steps
+// (more than one 32-step phase) after it is written, and its slot is rewritten
+// kMwRing - 33 = 95 steps after the read.  Used when a group's rows exceed one
+// warp (m > 256, or wide planes) and to put more warps on few long groups (the
+// paper's shape).  Same circuits and wavefront as the single-warp kernel.
+constexpr int kMwLag = 64, kMwRing = 128, kMwSP = 16;  // boundary words per column (padded)
+
+// 4 warps per SMSP (128 registers) while R*S <= 44 planes of row state fit
+// without large spills; above that the register count decides.
+template <int S, int R, int W>
+constexpr int mw_min_blocks() { return R * S <= 44 ? 16 / W : 1; }
+
+template <int S, int R, int W, int CIRC, class K>
+__global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_mw_kernel(const SweepArgs a, const K k) {
+  constexpr int LR = 32 * R;
+  static_assert(S <= kMwSP, "boundary row holds up to 16 planes");
+  const int lane = threadIdx.x & 31;
+  const int wk = threadIdx.x >> 5;  // row block of this warp
+  const int64_t stream = blockIdx.x;
+  if (stream >= a.streams) return;  // uniform per block
+  const int64_t Gs = a.base + (stream < a.rem ? 1 : 0);
+  const int64_t gb = stream * a.base + (stream < a.rem ? stream : a.rem);
+
+  __shared__ __align__(16) uint32_t bring[W - 1][kMwRing][kMwSP];
+  __shared__ __align__(16) uint32_t bzero[kMwSP];
+  __shared__ uint2 xring[W][2][32][R];
+  if (threadIdx.x < kMwSP) bzero[threadIdx.x] = 0;
+  __syncthreads();
+
+  const uint32_t nz = opaque(lane != 0 ? 1u : 0u);
+  const int row0 = wk * LR + lane * R;
+  uint32_t kill[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) kill[r] = opaque(row0 + r >= a.m ? 0xFFFFFFFFu : 0u);
+  // lane 0 of warps > 0 reads the ring of warp wk-1 (mask keeps the others on
+  // the zero row); lane 31 of warps < W-1 writes its own ring
+  const bool reader = lane == 0 && wk > 0;
+  const uint32_t* rbase = reader ? &bring[wk - 1][0][0] : bzero;
+  const uint32_t rmask = reader ? uint32_t(kMwRing * kMwSP - 1) : 0u;
+  const bool writer = lane == 31 && wk + 1 < W;
+  uint32_t* wbase = &bring[wk < W - 1 ? wk : 0][0][0];
+  // ring offset (words) of my current column J: (J mod kMwRing) * kMwSP
+  uint32_t off = uint32_t(-(lane + wk * kMwLag)) * kMwSP;
+
+  uint32_t H[R][S], dtop[S], M[S];
+#pragma unroll
+  for (int i = 0; i < S; ++i) {
+    dtop[i] = 0;
+    M[i] = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) H[r][i] = 0;
+  }
+  uint2 (*ring)[32][R] = xring[wk];
+  uint32_t xh[R], xl[R];
+  auto fetch_x = [&](int64_t gidx, int slot) {
+    int64_t g = gb + gidx;
+    g = g < a.G ? g : a.G - 1;
+    const uint2* xp = a.Xp + g * a.m + row0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) cp_async8(&ring[slot][lane][r], xp + r);
+    cp_async_commit();
+  };
+  fetch_x(0, 0);
+#pragma unroll
+  for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
+  const uint2* yp = a.Yp + gb * a.n - lane - wk * kMwLag;
+  int cnt = lane + wk * kMwLag;
+  int64_t gi = -1;
+  uint32_t flag = 0;
+
+  auto step = [&](const uint2 y) {
+    uint32_t up[S];
+    {
+      const uint4* b4 = reinterpret_cast<const uint4*>(rbase + (off & rmask));
+#pragma unroll
+      for (int q = 0; q < (S + 3) / 4; ++q) {
+        const uint4 v = b4[q];
+        const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (4 * q + e < S)
+            up[4 * q + e] = mad_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][4 * q + e], 1), nz, w[e]);
+      }
+    }
+    if (cnt == 0) {  // column 0 of my next group (divergent, once per group)
+      if (gi >= 0 && gi < Gs) {
+        if constexpr (BPBC_MODE == kModeThreshold) {
+          a.Mpart[((gb + gi) * W + wk) * 32 + lane] = flag;
+        } else {
+          uint32_t* dst = a.Mpart + (((gb + gi) * W + wk) * 32 + lane) * S;
+          if constexpr (CIRC == kExact) {
+            uint32_t F[S];
+            finish_exact<S, K::g>(M, F);
+#pragma unroll
+            for (int i = 0; i < S; ++i) dst[i] = F[i];
+          } else {
+#pragma unroll
+            for (int i = 0; i < S; ++i) dst[i] = M[i];
+          }
+        }
+      }
+      ++gi;
+      flag = 0;
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        M[i] = 0;
+        dtop[i] = 0;
+#pragma unroll
+        for (int r = 0; r < R; ++r) H[r][i] = 0;
+      }
+      cp_async_wait_all();
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const uint2 v = ring[gi & 1][lane][r];
+        xh[r] = v.x;
+        xl[r] = v.y;
+      }
+      fetch_x(gi + 1, int((gi + 1) & 1));
+      cnt = a.n;
+    }
+    --cnt;
+    uint32_t dg[S], u[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      dg[i] = dtop[i];
+      u[i] = up[i];
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      uint32_t hn[S], dn[S];
+      if constexpr (CIRC == kExact) {
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn);
+      } else {
+        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
+      }
+      if constexpr (BPBC_MODE == kModeThreshold) {
+        flag_gt<S, true>(flag, dn, a.tmask, kill[r]);
+      } else {
+        runmax<S, true>(M, dn, kill[r]);
+      }
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        dg[i] = H[r][i];
+        H[r][i] = hn[i];
+        u[i] = hn[i];
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < S; ++i) dtop[i] = up[i];
+    if (writer) {  // my bottom row at this column, for the next warp's lane 0
+      uint4* d4 = reinterpret_cast<uint4*>(wbase + (off & uint32_t(kMwRing * kMwSP - 1)));
+#pragma unroll
+      for (int q = 0; q < (S + 3) / 4; ++q) {
+        uint4 v;
+        v.x = 4 * q + 0 < S ? H[R - 1][4 * q + 0] : 0u;
+        v.y = 4 * q + 1 < S ? H[R - 1][4 * q + 1] : 0u;
+        v.z = 4 * q + 2 < S ? H[R - 1][4 * q + 2] : 0u;
+        v.w = 4 * q + 3 < S ? H[R - 1][4 * q + 3] : 0u;
+        d4[q] = v;
+      }
+    }
+    off += kMwSP;
+  };
+
+  uint2 y0 = __ldg(yp), y1;
+  for (int64_t tau = 0; tau < a.steps; tau += 32) {
+#pragma unroll 1
+    for (int i = 0; i < 32; i += 2) {
+      y1 = __ldg(yp + tau + i + 1);
+      step(y0);
+      y0 = __ldg(yp + tau + i + 2);
+      step(y1);
+    }
+    __syncthreads();  // phase boundary: ring writes of this phase -> reads of the next
+  }
+}
+
+template <int S, int R, int W, int CIRC, class K>
+void launch_mw(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
+  if constexpr (K::kFixed) {
+    sw_sweep_mw_kernel<S, R, W, CIRC, K><<<grid, block, 0, st>>>(a, K{});
+  } else {
+    sw_sweep_mw_kernel<S, R, W, CIRC, KRun><<<grid, block, 0, st>>>(a, kr);
+  }
+}
+
+template <int S, int MV>
+void reg_mw(SweepEntry (*mtab)[3][13]) {
+  constexpr int R = kMwR[MV], W = kMwW[MV];
+  using K211 = KFix<2, 1, 1>;
+  mtab[MV][0][S - 4] = {&launch_mw<S, R, W, kExact, K211>,
+                        (const void*)&sw_sweep_mw_kernel<S, R, W, kExact, K211>};
+  mtab[MV][1][S - 4] = {&launch_mw<S, R, W, kSat, K211>,
+                        (const void*)&sw_sweep_mw_kernel<S, R, W, kSat, K211>};
+  mtab[MV][2][S - 4] = {&launch_mw<S, R, W, kSat, KRun>,
+                        (const void*)&sw_sweep_mw_kernel<S, R, W, kSat, KRun>};
+}
+
 template <int S, int R, int L, int CIRC, bool PAD, class K>
 void launch_sweep(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
   if constexpr (K::kFixed) {
@@ -453,7 +657,12 @@ void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
 #define BPBC_CAT2(a, b) a##b
 #define BPBC_CAT(a, b) BPBC_CAT2(a, b)
 #define BPBC_REGNAME BPBC_CAT(BPBC_CAT(BPBC_CAT(register_sweep_s, BPBC_S), _m), BPBC_MODE)
-void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13]) {
+void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13],
+                  SweepEntry (*mtab)[3][13]) {
+  reg_mw<BPBC_S, 0>(mtab);
+  reg_mw<BPBC_S, 1>(mtab);
+  reg_mw<BPBC_S, 2>(mtab);
+  reg_mw<BPBC_S, 3>(mtab);
   reg_rl<BPBC_S, 0, false>(tab);
   reg_rl<BPBC_S, 1, false>(tab);
   reg_rl<BPBC_S, 2, false>(tab);
@@ -463,7 +672,6 @@ void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13]) {
   reg_rl<BPBC_S, 2, true>(tab);
   reg_rl<BPBC_S, 3, true>(tab);
   reg_striped<BPBC_S, 0>(stab);
-  reg_striped<BPBC_S, 1>(stab);
 }
 
 }  // namespace bpbc

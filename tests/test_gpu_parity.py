@@ -371,3 +371,35 @@ def test_filter_threshold_edges():
     with pytest.raises(bpbc.BPBCError) as ei:
         bpbc.filter_batch(dq, dt, -1, score_bits=8)
     assert ei.value.status == _lib.BPBC_ERR_INVALID_ARG
+
+
+# ---------------------------------------------------------------- wordwise comparator (NEXT-4)
+
+
+@pytest.mark.parametrize("P,m,n", [(1, 1, 1), (33, 9, 5), (1000, 40, 56), (4096, 128, 128),
+                                   (777, 256, 300), (500, 64, 1024), (301, 200, 90), (64, 32, 32)])
+def test_wordwise_matches_oracle(P, m, n):
+    q, t = synth.gen_pairs(9191 + m + n, P, m, n, planted=True)
+    dq = torch.from_numpy(q).to(DEV)
+    dt = torch.from_numpy(t).to(DEV)
+    got = bpbc.score_batch_wordwise(dq, dt, 2, -1, -1).cpu().numpy()
+    np.testing.assert_array_equal(got, oracle.sw_batch(q, t, 2, -1, -1))
+
+
+@pytest.mark.parametrize("consts", [(1, -1, -1), (3, -2, -1), (1, 0, 0), (5, -3, -4), (2, -7, -1)])
+def test_wordwise_runtime_constants(consts):
+    q, t = synth.gen_pairs(9292, 300, 37, 61, planted=True)
+    c1, mm, g = consts
+    got = bpbc.score_batch_wordwise(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV),
+                                    c1, mm, g).cpu().numpy()
+    np.testing.assert_array_equal(got, oracle.sw_batch(q, t, c1, mm, g))
+
+
+def test_wordwise_agrees_with_bitwise_at_c2_size():
+    """The two independent GPU algorithms agree on a full C2-sized batch."""
+    q, t = synth.gen_pairs(synth.seed_for_config(2), 1 << 20, 128, 128)
+    dq = torch.from_numpy(q).to(DEV)
+    dt = torch.from_numpy(t).to(DEV)
+    a = bpbc.score_batch_wordwise(dq, dt, 2, -1, -1)
+    b = bpbc.score_batch(dq, dt, 2, -1, -1, score_bits=9)
+    assert torch.equal(a, b)
