@@ -110,13 +110,17 @@ Layout layout(int64_t P, int mq, int nt) {
   Layout L;
   L.G = (P + 31) / 32;
   // room for the striped kernel whenever the plan may pick it (m > 128)
-  // room for the striped / multi-warp kernels' partials: 32 lanes per 64 rows
-  L.stripes = (mq + kMinStripeRows - 1) / kMinStripeRows;
+  // room for the striped / multi-warp kernels' partials: 32 lanes per 128 rows
+  // (per 64 rows when the opt-in few-groups split may use R = 2 warps)
+  const int rows_per_slot = getenv("BPBC_SPLIT_FEW_GROUPS") ? kMinStripeRows : 128;
+  L.stripes = (mq + rows_per_slot - 1) / rows_per_slot;
+  // the global boundary buffer is only used by the sequential striped kernel
+  const bool may_stripe = mq > 512 || (mq > 128 && getenv("BPBC_NO_MULTIWARP"));
   const int64_t xbytes = (L.G * mq + kXBackPad) * 8;
   const int64_t ybytes = (kYFrontPad + L.G * nt + nt + kYBackPadExtra) * 8;
   const int64_t mpbytes = L.G * L.stripes * 32 * 16 * 4;
   int64_t bnd_bytes = 0;
-  if (L.stripes > 1) {
+  if (may_stripe) {
     const int64_t per_stream = int64_t(nt) * 16 * 4;  // [n][16 words] at most
     int64_t st = L.G < kMaxStripeStreams ? L.G : kMaxStripeStreams;
     if (st * per_stream > kMaxBoundaryBytes) st = kMaxBoundaryBytes / per_stream;
@@ -353,6 +357,7 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   const bool mw = dsp.mw >= 0;
   const int64_t segs = mw ? 1 : 32 / L;
   int64_t cap_streams = dsp.cap_streams;
+  if (striped && lay.bnd_streams < 1) return BPBC_ERR_UNSUPPORTED;  // (layout/plan mismatch)
   if (striped && cap_streams > lay.bnd_streams) cap_streams = lay.bnd_streams;
   SweepArgs a;
   a.Xp = Xp;
