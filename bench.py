@@ -226,10 +226,21 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    ngpu = torch.cuda.device_count()
+    # More ranks than GPUs (only for exercising the N > 1 code path on a
+    # 1-GPU box): ranks share devices and the collectives go through gloo on
+    # the host; the timing is then not a scaling measurement.
+    shared = world > ngpu
+    if shared:
+        local = local % max(1, ngpu)
     if world > 1:
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
+    cdev = torch.device("cpu") if shared else dev  # where collective tensors live
     torch.cuda.set_device(dev)
     m, n, s = cfg["m"], cfg["n"], cfg["s"]
     seed = synth.seed_for_config(args.config)
@@ -284,7 +295,7 @@ def main():
     bpbc.profile(False, local)
     t_ms = sum(a.elapsed_time(b) for a, b in zip(starts, ends))
     if world > 1:
-        tt = torch.tensor([t_ms], dtype=torch.float64, device=dev)
+        tt = torch.tensor([t_ms], dtype=torch.float64, device=cdev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t_ms = tt.item()
     cells = P_total * m * n * args.steps
@@ -325,7 +336,6 @@ def main():
     # ---------------- wordwise comparator (NEXT-4) on the same resident batch
     wordwise = None
     if not args.no_filter and min(m, n) <= 256:
-        wws = torch.empty(max(ws.numel(), 1), dtype=torch.uint8, device=dev)
         wout = torch.empty(P, dtype=torch.int32, device=dev)
 
         def wstep():
@@ -352,7 +362,7 @@ def main():
                     "agrees_with_bitwise": agree,
                     "what": "bpbc_sw_score_batch_wordwise: ordinary-integer DP, 16-bit SIMD, "
                             "2 pairs per warp register (the paper's GPU wordwise row, P:L407)"}
-        del wws, wout
+        del wout
 
     # ---------------- end to end through the host-buffer C call
     e2e = e2e_packed2 = None
@@ -369,7 +379,7 @@ def main():
             bpbc.score_batch_host(qn, tn, *CONSTS, score_bits=s, device=local, out=on)
         el = time.perf_counter() - t0
         if world > 1:
-            te = torch.tensor([el], dtype=torch.float64, device=dev)
+            te = torch.tensor([el], dtype=torch.float64, device=cdev)
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
             el = te.item()
         e2e = {"value": round(P_total * m * n * ksteps / el / 1e9, 2), "unit": "GCUPS",
@@ -393,7 +403,7 @@ def main():
                                           out=on)
         el2 = time.perf_counter() - t0
         if world > 1:
-            te = torch.tensor([el2], dtype=torch.float64, device=dev)
+            te = torch.tensor([el2], dtype=torch.float64, device=cdev)
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
             el2 = te.item()
         e2e_packed2 = {"value": round(P_total * m * n * ksteps / el2 / 1e9, 2), "unit": "GCUPS",
@@ -404,7 +414,7 @@ def main():
 
     # ---------------- result gather (outside the timed region) + parity sample
     if world > 1:  # rank r holds the pairs of shard_range(P_total, world, r)
-        full = parallel.gather_scores(out, P_total)
+        full = parallel.gather_scores(out.to(cdev), P_total)
         got_all = full.cpu().numpy()
     else:
         got_all = out.cpu().numpy()
@@ -465,7 +475,10 @@ def main():
             "dtype": "u32 bit-sliced (s-bit scores)",
             "data": "synthetic (seeded i.i.d. uniform DNA, SplitMix64)",
             "config": {"workload": workload_name(args.config, cfg), "pairs_per_gpu": P, "pairs_total": P_total,
-                       "m": m, "n": n, "score_bits": s, "parallelism": f"dp{world} (pair shards)",
+                       "m": m, "n": n, "score_bits": s,
+                       "parallelism": f"dp{world} (pair shards)" + (
+                           f" on {ngpu} shared GPU(s): code-path check, not a scaling number"
+                           if shared else ""),
                        "l2": "inputs 320 MiB > 126 MB L2, plus a 256 MiB L2 flush between steps",
                        "plan": plan},
             "e2e": e2e, "e2e_packed2": e2e_packed2, "filter": filt, "wordwise": wordwise, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,

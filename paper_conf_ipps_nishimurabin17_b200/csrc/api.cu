@@ -114,6 +114,7 @@ Layout layout(int64_t P, int mq, int nt) {
   // (per 64 rows when the opt-in few-groups split may use R = 2 warps)
   const int rows_per_slot = getenv("BPBC_SPLIT_FEW_GROUPS") ? kMinStripeRows : 128;
   L.stripes = (mq + rows_per_slot - 1) / rows_per_slot;
+  if (L.stripes == 3) L.stripes = 4;  // multi-warp W = 3 runs as W = 4
   // the global boundary buffer is only used by the sequential striped kernel
   const bool may_stripe = mq > 512 || (mq > 128 && getenv("BPBC_NO_MULTIWARP"));
   const int64_t xbytes = (L.G * mq + kXBackPad) * 8;
@@ -223,7 +224,7 @@ int pick_mw(int mq, const Plan& p, int64_t G, int64_t short_cap) {
     return -1;
   };
   if (p.rl < 0) {  // the plan wants stripes
-    if (mq <= 512) return idx(4, (mq + 127) / 128 < 2 ? 2 : (mq + 127) / 128);
+    if (mq <= 512) return idx(4, (mq + 127) / 128 <= 2 ? 2 : 4);  // W = 3 runs as 4
     return -1;
   }
   // Few long groups (the paper's shape, G = 1024): splitting 128 rows over
@@ -342,6 +343,16 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   uint2* Yp = Ybase + kYFrontPad;
   uint32_t* Mpart = reinterpret_cast<uint32_t*>(ws + lay.mp_off);
 
+  // The sweep reads the pads around the planes (columns before / after a
+  // stream's groups, rows past m) and discards what it computes from them;
+  // zero them so those reads are of initialised memory.
+  {
+    cudaError_t ez = cudaMemsetAsync(Ybase, 0, size_t(kYFrontPad) * 8, st);
+    if (ez == cudaSuccess)
+      ez = cudaMemsetAsync(Yp + lay.G * nt, 0, size_t(nt + kYBackPadExtra) * 8, st);
+    if (ez == cudaSuccess) ez = cudaMemsetAsync(Xp + lay.G * mq, 0, size_t(kXBackPad) * 8, st);
+    if (ez != cudaSuccess) return cuda_fail(ctx, ez, "memset(pads)");
+  }
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
   if (ctx->profiling)
     for (int i = 0; i < 4; ++i) ev[i] = ctx->take_event();

@@ -174,6 +174,8 @@ cudaError_t launch_wordwise(const uint8_t* q, const uint8_t* t, int64_t P, int m
   a.rem = a.units % a.streams;
   a.steps = (a.base + (a.rem > 0 ? 1 : 0)) * int64_t(nt) + 32;
   const int grid = int((a.streams + 3) / 4);
+  e = cudaMemsetAsync(const_cast<uint8_t*>(a.dummy), 0, 256, st);  // read by idle lanes
+  if (e != cudaSuccess) return e;
   fns[R](a, grid, st);
   e = cudaGetLastError();
   if (e != cudaSuccess) return e;

@@ -1,0 +1,77 @@
+#!/usr/bin/env python3
+"""Small runs of every kernel family, for compute-sanitizer.
+
+    compute-sanitizer --tool memcheck|racecheck|synccheck python tools/sanitize_run.py
+
+Each case is small (sanitizers slow kernels ~100x) but spans several groups,
+ragged pair counts and ragged lengths: the single-warp sweep (L = 16 and 32,
+exact / saturating / runtime constants), the multi-warp sweep (shared-memory
+boundary ring + phase barriers), the sequential striped sweep (global boundary
+buffer), the threshold filter with compaction, the 2-bit packed input, the
+wordwise comparator and the host path.  Every result is checked against the
+oracle; exits non-zero on a mismatch.
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import oracle  # noqa: E402
+import synth  # noqa: E402
+import paper_conf_ipps_nishimurabin17_b200 as bpbc  # noqa: E402
+
+DEV = "cuda:0"
+
+
+def check(name, got, want):
+    bad = int((np.asarray(got) != np.asarray(want)).sum())
+    print(f"{name}: {'ok' if bad == 0 else f'{bad} MISMATCHES'}", flush=True)
+    return bad
+
+
+def main():
+    bad = 0
+    cases = [  # P, m, n, consts, s
+        (97, 64, 80, (2, -1, -1), None),      # L = 16, exact
+        (70, 128, 128, (2, -1, -1), None),    # L = 32, exact
+        (40, 200, 230, (2, -1, -1), None),    # R = 8
+        (50, 37, 61, (3, -2, -1), 12),        # runtime constants
+        (50, 48, 80, (2, -1, -1), 5),         # saturating, fixed constants
+        (33, 300, 320, (2, -1, -1), None),    # multi-warp W = 3 -> 4
+        (20, 200, 240, (31, -1, -1), 13),     # multi-warp wide planes
+        (9, 600, 640, (2, -1, -1), None),     # sequential stripes
+    ]
+    for P, m, n, (c1, mm, g), s in cases:
+        q, t = synth.gen_pairs(4000 + m + n, P, m, n, planted=True)
+        s = s or bpbc.default_score_bits(c1, m, n)
+        got = bpbc.score_batch(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV), c1, mm, g,
+                               score_bits=s).cpu().numpy()
+        bad += check(f"score P={P} m={m} n={n} c={c1},{mm},{g} s={s} plan={bpbc.last_plan(0)}",
+                     got, oracle.sw_batch(q, t, c1, mm, g, score_bits=s))
+    # threshold filter with compaction
+    q, t = synth.gen_pairs(77, 150, 64, 96, planted=True)
+    mask, count, idx = bpbc.filter_batch(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV), 40)
+    want = np.nonzero(oracle.sw_batch(q, t, 2, -1, -1) > 40)[0]
+    c = int(count.item())
+    bad += check("filter indices", idx.cpu().numpy()[:c], want)
+    # packed2 input, wordwise comparator, host path
+    q, t = synth.gen_pairs(78, 90, 72, 100, planted=True)
+    want = oracle.sw_batch(q, t, 2, -1, -1, score_bits=9)
+    got = bpbc.score_batch_packed2(torch.from_numpy(synth.pack2bit(q)).to(DEV),
+                                   torch.from_numpy(synth.pack2bit(t)).to(DEV), 72, 100,
+                                   score_bits=9).cpu().numpy()
+    bad += check("packed2", got, want)
+    got = bpbc.score_batch_wordwise(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV)).cpu()
+    bad += check("wordwise", got.numpy(), oracle.sw_batch(q, t, 2, -1, -1))
+    bad += check("host path", bpbc.score_batch_host(q, t, 2, -1, -1, 9), want)
+    torch.cuda.synchronize()
+    print("sanitize_run:", "PASS" if bad == 0 else "FAIL", flush=True)
+    sys.exit(1 if bad else 0)
+
+
+if __name__ == "__main__":
+    main()
