@@ -482,8 +482,9 @@ def main():
                        "l2": "inputs 320 MiB > 126 MB L2, plus a 256 MiB L2 flush between steps",
                        "plan": plan},
             "e2e": e2e, "e2e_packed2": e2e_packed2, "filter": filt, "wordwise": wordwise, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,
-            # ours per step and rank: pack (query+target), sweep, extract
-            "gpu_launches": 3 * args.steps * world, "parity": parity}
+            # ours per step and rank, from the library (fused sweep + extract,
+            # or pack + sweep + extract)
+            "gpu_launches": plan["kernels"] * args.steps * world, "parity": parity}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

@@ -232,6 +232,13 @@ int bpbc_sw_get_error_flags(bpbc_sw_ctx *ctx, uint32_t *flags);
 int bpbc_sw_last_plan(bpbc_sw_ctx *ctx, int32_t *circuit, int32_t *width, int32_t *rows_per_lane,
                       int32_t *lanes, int64_t *streams, int32_t *ops_per_word_cell);
 
+/* Kernels of this library the last bpbc_sw_score_batch / _filter_batch call
+ * on this ctx launched (pack, sweep, epilogue kernels; the CUB scan of the
+ * filter compaction counts as one), and whether its sweep was the fused
+ * kernel that transposes the raw codes itself (1) or ran on packed planes
+ * (0).  Either pointer may be NULL. */
+int bpbc_sw_last_launches(bpbc_sw_ctx *ctx, int32_t *kernels, int32_t *fused);
+
 /* Per-phase device timing, the columns of the paper's Table IV (P:L384-413:
  * W2B, SWA, B2W).  bpbc_sw_profile(ctx, 1) clears the accumulators and makes
  * every following bpbc_sw_score_batch* call record CUDA events around its

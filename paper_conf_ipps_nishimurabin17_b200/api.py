@@ -262,9 +262,12 @@ def last_plan(device: int = 0) -> dict:
     check(_lib.load().bpbc_sw_last_plan(_ctx(device), ctypes.byref(c), ctypes.byref(w),
                                         ctypes.byref(r), ctypes.byref(l), ctypes.byref(s),
                                         ctypes.byref(o)))
+    k, f = ctypes.c_int32(), ctypes.c_int32()
+    check(_lib.load().bpbc_sw_last_launches(_ctx(device), ctypes.byref(k), ctypes.byref(f)))
     return {"circuit": ["exact", "saturating"][c.value] if c.value >= 0 else None,
             "width": w.value, "rows_per_lane": r.value, "lanes": l.value,
-            "streams": s.value, "ops_per_word_cell": o.value}
+            "streams": s.value, "ops_per_word_cell": o.value, "kernels": k.value,
+            "fused": bool(f.value)}
 
 
 def profile(enable: bool, device: int = 0) -> None:

@@ -31,6 +31,7 @@ struct bpbc_sw_ctx {
   char err[512] = {0};
   // last plan
   int32_t plan_circuit = -1, plan_width = 0, plan_R = 0, plan_L = 0, plan_ops = 0;
+  int32_t plan_kernels = 0, plan_fused = 0;  // kernels the last call launched; fused sweep?
   int64_t plan_streams = 0;
   // phase profiling (bpbc_sw_profile): 4 events per recorded call
   bool profiling = false;
@@ -56,15 +57,17 @@ namespace {
 SweepEntry g_table[2][kNumVariants][kNumRL][13];  // [mode][variant][rl][S - 4]
 SweepEntry g_striped[2][kNumStripeRV][3][13];     // [mode][stripe R][kind][S - 4]
 SweepEntry g_mw[2][kNumMw][3][13];                // [mode][(R, W)][kind][S - 4]
+SweepEntry g_planes[2][kNumVariants][2][13];      // [mode][variant][rl 0..1][S - 4]
 std::once_flag g_table_once;
 
 void init_table() {
   memset(g_table, 0, sizeof(g_table));
   memset(g_striped, 0, sizeof(g_striped));
   memset(g_mw, 0, sizeof(g_mw));
+  memset(g_planes, 0, sizeof(g_planes));
 #define BPBC_REG(S)                                      \
-  register_sweep_s##S##_m0(g_table[0], g_striped[0], g_mw[0]); \
-  register_sweep_s##S##_m1(g_table[1], g_striped[1], g_mw[1]);
+  register_sweep_s##S##_m0(g_table[0], g_striped[0], g_mw[0], g_planes[0]); \
+  register_sweep_s##S##_m1(g_table[1], g_striped[1], g_mw[1], g_planes[1]);
   BPBC_REG(4)
   BPBC_REG(5)
   BPBC_REG(6)
@@ -210,6 +213,7 @@ struct Dispatch {
   Plan plan;
   SweepEntry ent;
   bool striped;
+  bool fused = false;   // single-warp kernel reading raw codes (no pack pass)
   int mw = -1;          // multi-warp variant (index into kMwR / kMwW), -1 = none
   int R, L, W = 1;      // rows per lane, lanes per group, warps per group
   int64_t cap_streams;  // resident streams (before the boundary-buffer cap)
@@ -262,7 +266,7 @@ int occupancy_blocks(const void* func) {  // cached per kernel
   return nb;
 }
 
-int make_dispatch(bpbc_sw_ctx* ctx, int mq, int c1, int c2, int g, int S, Dispatch* d,
+int make_dispatch(bpbc_sw_ctx* ctx, int mq, int nt, int c1, int c2, int g, int S, Dispatch* d,
                   int mode = kModeMax, int64_t G = 0) {
   int rc = make_plan(mq, c1, c2, g, S, &d->plan);
   if (rc != BPBC_OK) return rc;
@@ -275,6 +279,16 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int c1, int c2, int g, int S, Dispat
                           [plan.width - 4]
                : g_table[mode][variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl]
                         [plan.width - 4];
+  // single-warp plans: the fused kernel unless the target is too short for
+  // its phase-granular query transposes (n < L + 32, only for L = 16)
+  if (!d->striped) {
+    d->fused = nt >= kRLL[plan.rl] + 32;
+    if (!d->fused) {
+      if (plan.rl > 1) return BPBC_ERR_UNSUPPORTED;  // (cannot happen: n >= m > 64)
+      d->ent = g_planes[mode][variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl]
+                       [plan.width - 4];
+    }
+  }
   if (!d->ent.launch) return BPBC_ERR_UNSUPPORTED;
   d->R = d->striped ? kStripeRV[plan.stripe_rv] : kRLR[plan.rl];
   d->L = d->striped ? 32 : kRLL[plan.rl];
@@ -290,6 +304,7 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int c1, int c2, int g, int S, Dispat
     if (e.launch) {
       d->ent = e;
       d->striped = false;
+      d->fused = false;
       d->R = kMwR[d->mw];
       d->W = kMwW[d->mw];
       d->L = 32;
@@ -334,7 +349,7 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   }
   const int c1 = match, c2 = -mismatch, g = -gap;
   Dispatch dsp;
-  int rc = make_dispatch(ctx, mq, c1, c2, g, S, &dsp, o.mode, (P + 31) / 32);
+  int rc = make_dispatch(ctx, mq, nt, c1, c2, g, S, &dsp, o.mode, (P + 31) / 32);
   if (rc != BPBC_OK) return rc;
   const Plan& plan = dsp.plan;
   const Layout lay = layout(P, mq, nt);
@@ -357,9 +372,11 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   if (ctx->profiling)
     for (int i = 0; i < 4; ++i) ev[i] = ctx->take_event();
   if (ev[0]) cudaEventRecord(ev[0], st);
-  cudaError_t e =
-      launch_pack2(qx, mq, Xp, ty, nt, Yp, P, ctx->d_flags, ctx->num_sms, st, packed2);
-  if (e != cudaSuccess) return cuda_fail(ctx, e, "pack");
+  cudaError_t e = cudaSuccess;
+  if (!dsp.fused) {  // the fused kernel transposes the raw codes itself
+    e = launch_pack2(qx, mq, Xp, ty, nt, Yp, P, ctx->d_flags, ctx->num_sms, st, packed2);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "pack");
+  }
 
   if (ev[1]) cudaEventRecord(ev[1], st);
   const bool striped = dsp.striped;
@@ -401,12 +418,19 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   a.base = lay.G / a.streams;
   a.rem = lay.G % a.streams;
   a.stripes = striped ? (mq + 32 * R - 1) / (32 * R) : 1;
+  a.qraw = qx;
+  a.traw = ty;
+  a.qstride = packed2 ? (int64_t(mq) + 3) / 4 : mq;
+  a.tstride = packed2 ? (int64_t(nt) + 3) / 4 : nt;
+  a.P = P;
+  a.packed2 = packed2 ? 1 : 0;
+  a.flags = ctx->d_flags;
   a.bnd = reinterpret_cast<uint32_t*>(ws + lay.bnd_off);
   a.bzero = reinterpret_cast<const uint32_t*>(ws + lay.zero_off);
   a.steps = (a.base + (a.rem > 0 ? 1 : 0)) * a.stripes * int64_t(nt) + L;
   if (mw) a.steps += int64_t(W - 1) * 64 + 31;  // warp lag (kMwLag), then whole phases
   a.steps += a.steps & 1;  // the short kernel runs two steps per iteration
-  if (mw) a.steps = (a.steps + 31) / 32 * 32;
+  if (mw || dsp.fused) a.steps = (a.steps + 31) / 32 * 32;  // whole 32-step phases
   if (striped) {
     e = cudaMemsetAsync(ws + lay.zero_off, 0, 256, st);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "memset(zero row)");
@@ -448,6 +472,10 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   ctx->plan_L = L * W;  // lanes per group (over all its warps)
   ctx->plan_ops = plan.ops;
   ctx->plan_streams = a.streams;
+  ctx->plan_fused = dsp.fused ? 1 : 0;
+  ctx->plan_kernels = (dsp.fused ? 0 : 1) + 1 + (o.mode == kModeThreshold
+                                                     ? ((o.indices || o.count) ? 2 : 1)
+                                                     : 1);
   return BPBC_OK;
 }
 
@@ -550,7 +578,8 @@ int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t*
   // stream of a chunk gets the same number of groups), growing 1, 2, 4, ...
   // waves: the first copy is short, later chunks amortise the pipeline fill.
   Dispatch dsp;
-  rc = make_dispatch(ctx, m < n ? m : n, match, -mismatch, -gap, score_bits, &dsp);
+  rc = make_dispatch(ctx, m < n ? m : n, m < n ? n : m, match, -mismatch, -gap, score_bits,
+                     &dsp);
   if (rc != BPBC_OK) return rc;
   const int64_t wave_pairs = dsp.cap_streams * 32;
   // copy-bound (u8 rows: ~1 byte per base vs ~50 GB/s H2D) -> equal chunks so
@@ -845,6 +874,13 @@ int bpbc_sw_last_plan(bpbc_sw_ctx* ctx, int32_t* circuit, int32_t* width, int32_
   if (lanes) *lanes = ctx->plan_L;
   if (streams) *streams = ctx->plan_streams;
   if (ops_per_word_cell) *ops_per_word_cell = ctx->plan_ops;
+  return BPBC_OK;
+}
+
+int bpbc_sw_last_launches(bpbc_sw_ctx* ctx, int32_t* kernels, int32_t* fused) {
+  if (!ctx) return BPBC_ERR_INVALID_ARG;
+  if (kernels) *kernels = ctx->plan_kernels;
+  if (fused) *fused = ctx->plan_fused;
   return BPBC_OK;
 }
 

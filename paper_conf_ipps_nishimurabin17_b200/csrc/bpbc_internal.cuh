@@ -36,6 +36,14 @@ struct SweepArgs {
   int64_t rem;       //   (the first rem streams get base+1)
   int64_t steps;     // wavefront steps = (base + (rem>0)) * stripes * n + L
   // long-query (striped) kernel only
+  // fused single-warp kernel: the caller's raw codes (query rows m, target
+  // rows n, after the R17 swap), u8 or 2-bit packed
+  const uint8_t* qraw;
+  const uint8_t* traw;
+  int64_t qstride, tstride;  // bytes per row
+  int64_t P;                 // pairs (rows of qraw / traw)
+  int packed2;
+  uint32_t* flags;           // sticky error flags (bad base codes)
   // threshold mode (bpbc_sw_filter_batch): bits of the compared threshold as
   // all-ones / all-zeros masks (tau + g for the exact circuit, tau otherwise)
   uint32_t tmask[16];
@@ -75,9 +83,9 @@ SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
 // (+2,-1,-1), 2 saturating runtime constants).
 #define BPBC_DECLARE_REG(S)                                                       \
   void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13], \
-                                SweepEntry (*mtab)[3][13]);                               \
+                                SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]);    \
   void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13], \
-                                SweepEntry (*mtab)[3][13]);
+                                SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]);
 BPBC_DECLARE_REG(4)
 BPBC_DECLARE_REG(5)
 BPBC_DECLARE_REG(6)

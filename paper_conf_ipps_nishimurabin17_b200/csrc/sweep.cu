@@ -26,6 +26,7 @@
 //     its state in a short divergent branch taken once per group per lane;
 //   * the cell is a fixed LOP3 circuit (circuit.cuh): no branch on data.
 #include "bpbc_internal.cuh"
+#include "transpose.cuh"
 
 #ifndef BPBC_S
 #error "compile with -DBPBC_S=<score width>"
@@ -58,8 +59,267 @@ __device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
+// Target chunk that straddles two groups of a stream (only when n % 32 != 0):
+// lane k gathers positions col.. of pair 32g+k, continuing into pair
+// 32(g+1)+k after the row end; folded H / L as tr_load_fold.  Out of line:
+// one copy per object instead of one per kernel instantiation.
+__device__ __noinline__ uint3 gather_straddle(const uint8_t* traw, int64_t tstride, int n,
+                                              int64_t P, int64_t g, bool has_next, int col,
+                                              int lane, bool packed2) {
+  uint32_t H, L, bad = 0;
+  uint32_t w[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  const int64_t row0 = g * 32 + lane, row1 = (g + 1) * 32 + lane;
+#pragma unroll
+  for (int i = 0; i < 32; ++i) {
+    const bool next = col + i >= n;  // past this group's last column
+    const int cc = col + i - (next ? n : 0);
+    const int64_t row = next ? row1 : row0;
+    uint32_t code = 0;
+    if ((next ? has_next : true) && row < P) {
+      code = packed2 ? (traw[row * tstride + cc / 4] >> (2 * (cc & 3))) & 3u
+                     : traw[row * tstride + cc];
+    }
+    if (packed2) {  // place as a 2-bit field of the packed layout
+      w[i >> 4] |= (code & 3u) << (2 * (i & 15));
+    } else {
+      w[i >> 2] |= (code & 0xFFu) << (8 * (i & 3));
+    }
+  }
+  if (packed2) tr_fold_packed2(w[0], w[1], H, L);
+  else tr_fold_u8(w, H, L, bad);
+  return make_uint3(H, L, bad);  // by value: registers, no stack frame at the call
+}
+
+// ---------------------------------------------------------------------------
+// The single-warp sweep with the W2B transpose fused in:
+// it reads the caller's raw codes (u8, or 2-bit packed) and builds the bit
+// planes itself, so no separate pack pass and no planes in HBM.
+//
+//   * target: every 32 steps (a "phase") the warp transposes the next 32
+//     columns of each segment's virtual target (tr_load_fold + tr_butterfly,
+//     transpose.cuh) into a shared-memory ring of 128 columns, stored twice
+//     (slots j and j + 128) so a lane's 32 reads of a phase never wrap; the
+//     ring holds chunks p-1..p+2 and chunk p+2 is built at the start of phase
+//     p, so reads never wait on it;
+//   * query: the planes of a segment's next group are transposed into a
+//     2-slot shared ring at a phase start after every lane has entered the
+//     current group (and before lane 0 leaves it: needs n >= L + 32);
+//   * a __syncwarp at each phase start orders the ring writes before reads.
 template <int S, int R, int L, int CIRC, bool PAD, class K>
 __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const K k) {
+  constexpr int SEGS = 32 / L;
+  constexpr int XCH = (L * R + 31) / 32;  // 32-row chunks of a group's query rows
+  const int lane = threadIdx.x & 31;
+  const int sl = lane & (L - 1);
+  const int seg = lane / L;
+  const int wib = threadIdx.x >> 5;
+  const int64_t warp = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  if (warp * SEGS >= a.streams) return;  // uniform per warp
+  const int64_t stream = warp * SEGS + seg;
+
+  // groups of segment s's stream (uniform per warp for each s)
+  auto seg_range = [&](int s, int64_t& gbs, int64_t& gss) {
+    const int64_t st = warp * SEGS + s;
+    gss = 0;
+    gbs = 0;
+    if (st < a.streams) {
+      gss = a.base + (st < a.rem ? 1 : 0);
+      gbs = st * a.base + (st < a.rem ? st : a.rem);
+    }
+  };
+  int64_t Gs, gb;
+  seg_range(seg, gb, Gs);
+  const uint32_t nz = opaque(sl != 0 ? 1u : 0u);
+  uint32_t kill[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) kill[r] = PAD ? opaque((sl * R + r >= a.m) ? 0xFFFFFFFFu : 0u) : 0u;
+
+  uint32_t H[R][S], dtop[S], M[S];
+#pragma unroll
+  for (int i = 0; i < S; ++i) {
+    dtop[i] = 0;
+    M[i] = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) H[r][i] = 0;
+  }
+  __shared__ uint2 xring[4][2][32][R];        // [warp][slot][lane][row]
+  __shared__ uint2 yring[4][SEGS][256];       // [warp][segment][column slot, doubled]
+  uint2 (*xr)[32][R] = xring[wib];
+  uint2 (*yr)[256] = yring[wib];
+  const bool packed2 = a.packed2 != 0;
+  const int mypos = packed2 ? tr_pos_packed2(lane) : tr_pos_u8(lane);
+  uint32_t bad = 0;
+
+  // target columns [32c, 32c + 32) of segment s's virtual target -> ring
+  auto build_y = [&](int s, int64_t c) {
+    int64_t gbs, gss;
+    seg_range(s, gbs, gss);
+    const int64_t v0 = 32 * c;  // first virtual column
+    uint32_t Hw = 0, Lw = 0;
+    if (v0 >= 0 && v0 < gss * a.n) {
+      const int64_t h = v0 / a.n;
+      const int col = int(v0 - h * a.n);
+      const int64_t g = gbs + h;
+      if (col + 32 <= a.n) {
+        tr_load_fold(a.traw, a.tstride, a.n, g * 32 + lane, a.P, col, packed2, Hw, Lw, bad);
+      } else {  // the chunk straddles two groups (n % 32 != 0; n >= 48)
+        const uint3 r3 = gather_straddle(a.traw, a.tstride, a.n, a.P, g, h + 1 < gss, col, lane,
+                                         packed2);
+        Hw = r3.x;
+        Lw = r3.y;
+        bad |= r3.z;
+      }
+    }
+    tr_butterfly(Hw, Lw, lane);
+    const int slot = int((v0 + mypos) & 127);
+    yr[s][slot] = make_uint2(Hw, Lw);
+    yr[s][slot + 128] = make_uint2(Hw, Lw);
+  };
+  // query rows of segment s's group h (stream-relative) -> x slot h & 1
+  auto build_x = [&](int s, int64_t h) {
+    int64_t gbs, gss;
+    seg_range(s, gbs, gss);
+    int64_t g = gbs + h;
+    g = g < a.G ? g : a.G - 1;
+#pragma unroll
+    for (int c = 0; c < XCH; ++c) {
+      uint32_t Hw = 0, Lw = 0;
+      tr_load_fold(a.qraw, a.qstride, a.m, g * 32 + lane, a.P, 32 * c, packed2, Hw, Lw, bad);
+      tr_butterfly(Hw, Lw, lane);
+      const int row = 32 * c + mypos;  // rows >= m are zero (tr_load_fold)
+      if (row < L * R) xr[int(h & 1)][s * L + row / R][row % R] = make_uint2(Hw, Lw);
+    }
+  };
+
+  uint32_t xh[R], xl[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
+  int cnt = sl;      // steps until my next group starts (J % n == 0)
+  int64_t gi = -1;   // my current group within the stream
+  uint32_t flag = 0; // threshold mode: pairs with a cell > tau so far
+
+  // One wavefront step with target planes y of my current column.
+  auto step = [&](const uint2 y) {
+    uint32_t up[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
+
+    if (cnt == 0) {  // column 0 of my next group (divergent, once per group)
+      if (gi >= 0 && gi < Gs) {
+        if constexpr (BPBC_MODE == kModeThreshold) {
+          a.Mpart[(gb + gi) * L + sl] = flag;  // one flag word per lane
+        } else {
+          uint32_t* dst = a.Mpart + ((gb + gi) * L + sl) * S;
+          if constexpr (CIRC == kExact) {
+            uint32_t F[S];
+            finish_exact<S, K::g>(M, F);  // M tracked D' = diag + w + g
+#pragma unroll
+            for (int i = 0; i < S; ++i) dst[i] = F[i];
+          } else {
+#pragma unroll
+            for (int i = 0; i < S; ++i) dst[i] = M[i];
+          }
+        }
+      }
+      ++gi;
+      flag = 0;
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        M[i] = 0;
+        dtop[i] = 0;
+#pragma unroll
+        for (int r = 0; r < R; ++r) H[r][i] = 0;
+      }
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const uint2 v = xr[int(gi & 1)][lane][r];
+        xh[r] = v.x;
+        xl[r] = v.y;
+      }
+      cnt = a.n;
+    }
+    --cnt;
+
+    uint32_t dg[S], u[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      dg[i] = dtop[i];
+      u[i] = up[i];
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      uint32_t hn[S], dn[S];
+      // running max over the diagonal term (circuit.cuh finish_exact); padded
+      // rows are masked out of it
+      if constexpr (CIRC == kExact) {
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn);
+      } else {
+        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
+      }
+      if constexpr (BPBC_MODE == kModeThreshold) {
+        flag_gt<S, PAD>(flag, dn, a.tmask, kill[r]);
+      } else {
+        runmax<S, PAD>(M, dn, kill[r]);
+      }
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        dg[i] = H[r][i];
+        H[r][i] = hn[i];
+        u[i] = hn[i];
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < S; ++i) dtop[i] = up[i];
+  };
+
+  // prologue: the first group's query planes, target chunks -1 (zeros), 0, 1
+#pragma unroll
+  for (int s = 0; s < SEGS; ++s) {
+    yr[s][lane] = yr[s][lane + 32] = yr[s][lane + 64] = yr[s][lane + 96] = make_uint2(0u, 0u);
+    yr[s][lane + 128] = yr[s][lane + 160] = yr[s][lane + 192] = yr[s][lane + 224] =
+        make_uint2(0u, 0u);
+  }
+  __syncwarp();
+  int64_t xnext[SEGS];
+#pragma unroll
+  for (int s = 0; s < SEGS; ++s) {
+    build_x(s, 0);
+    xnext[s] = 1;
+    build_y(s, 0);
+    build_y(s, 1);
+  }
+  const int64_t phases = a.steps / 32;  // a.steps is a multiple of 32
+  for (int64_t p = 0; p < phases; ++p) {
+    __syncwarp();  // this warp's ring writes of the previous phase -> reads
+#pragma unroll
+    for (int s = 0; s < SEGS; ++s) {
+      build_y(s, p + 2);
+      // group h's query may be written into slot h & 1 once every lane of
+      // the segment has entered group h - 1 (step (h-1) n + L); lane 0 needs
+      // it at step h n
+      if ((xnext[s] - 1) * a.n + L <= 32 * p) {
+        build_x(s, xnext[s]);
+        ++xnext[s];
+      }
+    }
+    __syncwarp();
+    const uint2* yb = &yr[seg][(32 * p - sl) & 127];  // my 32 columns of this phase
+#pragma unroll 1
+    for (int i = 0; i < 32; i += 2) {
+      const uint2 y0 = yb[i], y1 = yb[i + 1];
+      step(y0);
+      step(y1);
+    }
+  }
+  if (__any_sync(0xFFFFFFFFu, bad != 0) && lane == 0) atomicOr(a.flags, BPBC_FLAG_BAD_BASE);
+}
+
+// ---------------------------------------------------------------------------
+// The single-warp sweep on pre-packed planes (pack_kernel output): used when
+// the target is too short (n < L + 32) for the fused kernel's phase-granular
+// query transposes.  Same wavefront and circuits.
+template <int S, int R, int L, int CIRC, bool PAD, class K>
+__global__ void __launch_bounds__(128) sw_sweep_planes_kernel(const SweepArgs a, const K k) {
   constexpr int SEGS = 32 / L;
   const int lane = threadIdx.x & 31;
   const int sl = lane & (L - 1);
@@ -637,6 +897,30 @@ void reg_striped(SweepEntry (*stab)[3][13]) {
                         (const void*)&sw_sweep_striped_kernel<S, kSat, KRun, R>};
 }
 
+template <int S, int R, int L, int CIRC, bool PAD, class K>
+void launch_planes(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
+  if constexpr (K::kFixed) {
+    sw_sweep_planes_kernel<S, R, L, CIRC, PAD, K><<<grid, block, 0, st>>>(a, K{});
+  } else {
+    sw_sweep_planes_kernel<S, R, L, CIRC, PAD, KRun><<<grid, block, 0, st>>>(a, kr);
+  }
+}
+
+template <int S, int RL, bool PAD>
+void reg_planes(SweepEntry (*ptab)[2][13]) {
+  constexpr int R = kRLR[RL], L = kRLL[RL];
+  using K211 = KFix<2, 1, 1>;
+  ptab[variant_index(kExact, kC211, PAD)][RL][S - 4] = {
+      &launch_planes<S, R, L, kExact, PAD, K211>,
+      (const void*)&sw_sweep_planes_kernel<S, R, L, kExact, PAD, K211>};
+  ptab[variant_index(kSat, kC211, PAD)][RL][S - 4] = {
+      &launch_planes<S, R, L, kSat, PAD, K211>,
+      (const void*)&sw_sweep_planes_kernel<S, R, L, kSat, PAD, K211>};
+  ptab[variant_index(kSat, kCRun, PAD)][RL][S - 4] = {
+      &launch_planes<S, R, L, kSat, PAD, KRun>,
+      (const void*)&sw_sweep_planes_kernel<S, R, L, kSat, PAD, KRun>};
+}
+
 template <int S, int RL, bool PAD>
 void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
   constexpr int R = kRLR[RL], L = kRLL[RL];
@@ -658,7 +942,11 @@ void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
 #define BPBC_CAT(a, b) BPBC_CAT2(a, b)
 #define BPBC_REGNAME BPBC_CAT(BPBC_CAT(BPBC_CAT(register_sweep_s, BPBC_S), _m), BPBC_MODE)
 void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13],
-                  SweepEntry (*mtab)[3][13]) {
+                  SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]) {
+  reg_planes<BPBC_S, 0, false>(ptab);
+  reg_planes<BPBC_S, 1, false>(ptab);
+  reg_planes<BPBC_S, 0, true>(ptab);
+  reg_planes<BPBC_S, 1, true>(ptab);
   reg_mw<BPBC_S, 0>(mtab);
   reg_mw<BPBC_S, 1>(mtab);
   reg_mw<BPBC_S, 2>(mtab);

@@ -403,3 +403,30 @@ def test_wordwise_agrees_with_bitwise_at_c2_size():
     a = bpbc.score_batch_wordwise(dq, dt, 2, -1, -1)
     b = bpbc.score_batch(dq, dt, 2, -1, -1, score_bits=9)
     assert torch.equal(a, b)
+
+
+def test_c5_point_full_size_sampled():
+    """BASELINE config 5's largest point at full size: 2^22 pairs, m = n = 512,
+    11-bit slices (the multi-warp kernel), checked on a seeded sample."""
+    _sampled(5, 1 << 22, 512, 512, 11, sample=512)
+    assert bpbc.last_plan(0)["lanes"] == 128  # 4 warps x 32 lanes per group
+
+
+def test_filter_c2_full_size_sampled():
+    """Threshold filter at C2's size: the flagged set on a sample equals the
+    oracle's, and the count equals the number of set mask bits."""
+    P, m, n, tau = 1 << 20, 128, 128, 110
+    q, t = synth.gen_pairs(synth.seed_for_config(2), P, m, n, planted=True)
+    mask, count, idx = bpbc.filter_batch(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV),
+                                         tau, score_bits=9)
+    words = mask.cpu().numpy().view(np.uint32)
+    bits = ((words[:, None] >> np.arange(32, dtype=np.uint32)[None, :]) & 1).reshape(-1)
+    c = int(count.item())
+    assert c == int(bits.sum())
+    got_idx = idx.cpu().numpy()[:c]
+    assert np.all(np.diff(got_idx) > 0)
+    np.testing.assert_array_equal(got_idx, np.nonzero(bits)[0])
+    rng = np.random.default_rng(2)
+    sample = np.sort(rng.choice(P, size=4096, replace=False))
+    want = oracle.sw_batch(q[sample], t[sample], 2, -1, -1) > tau
+    np.testing.assert_array_equal(bits[sample].astype(bool), want)
