@@ -102,7 +102,7 @@ int cuda_fail(bpbc_sw_ctx* ctx, cudaError_t e, const char* what) {
 // offsets 256-byte aligned.
 struct Layout {
   int64_t G = 0;
-  int stripes = 1;             // > 1 only for the long-query (striped) kernel
+  int stripes = 1;             // 32-lane partial slots per group (multi-warp / striped)
   int64_t bnd_streams = 0;     // streams the boundary buffer has room for
   int64_t x_off = 0, y_off = 0, mp_off = 0, bnd_off = 0, zero_off = 0, total = 0;
 };
@@ -112,7 +112,6 @@ int64_t align256(int64_t v) { return (v + 255) & ~int64_t(255); }
 Layout layout(int64_t P, int mq, int nt) {
   Layout L;
   L.G = (P + 31) / 32;
-  // room for the striped kernel whenever the plan may pick it (m > 128)
   // room for the striped / multi-warp kernels' partials: 32 lanes per 128 rows
   // (per 64 rows when the opt-in few-groups split may use R = 2 warps)
   const int rows_per_slot = getenv("BPBC_SPLIT_FEW_GROUPS") ? kMinStripeRows : 128;
@@ -358,10 +357,10 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   uint2* Yp = Ybase + kYFrontPad;
   uint32_t* Mpart = reinterpret_cast<uint32_t*>(ws + lay.mp_off);
 
-  // The sweep reads the pads around the planes (columns before / after a
-  // stream's groups, rows past m) and discards what it computes from them;
-  // zero them so those reads are of initialised memory.
-  {
+  // The planes-reading sweeps read the pads around the planes (columns before
+  // / after a stream's groups, rows past m) and discard what they compute
+  // from them; zero them so those reads are of initialised memory.
+  if (!dsp.fused) {
     cudaError_t ez = cudaMemsetAsync(Ybase, 0, size_t(kYFrontPad) * 8, st);
     if (ez == cudaSuccess)
       ez = cudaMemsetAsync(Yp + lay.G * nt, 0, size_t(nt + kYBackPadExtra) * 8, st);
