@@ -207,7 +207,7 @@ BPBC_HD void ssub_run(const uint32_t (&X)[S], const uint32_t* gm, uint32_t (&U)[
 // (then no intermediate overflows and nothing goes negative):
 //   e  = (xH ^ yH) | (xL ^ yL)                  mismatch flag
 //   D' = diag + (e ? g - c2 : c1 + g)           one ripple adder
-//   X  = max(up, left, D')                      two max_B
+//   X  = max(up, max(left, D'))                 two max_B
 //   H  = max(X - g, 0)  = max(0, up-g, left-g, diag+w)
 // kill forces H = 0 (rows past m).  LOP3 per word-cell:
 //   2 + (2S - 1) + 4S + (2S - 1) = 8S, 10S with the running max
@@ -231,9 +231,13 @@ BPBC_HD void cell_exact(const uint32_t (&up)[S], const uint32_t (&left)[S],
     D[i] = lop3<kSumLit<kind>>(diag[i], e, c);
     if constexpr (i + 1 < S) c = lop3<kCarryLit<kind>>(diag[i], e, c);
   });
+  // X = max(up, max(left, D')): the inner max does not depend on `up` (the
+  // previous row's fresh output), so only one comparator + mux + the gap
+  // subtract sit on the row-to-row dependency chain (2S+1 deep instead of
+  // 3S+2); same gate count as max(max(up, left), D').
   uint32_t T[S], X[S];
-  mux<S>(lt<S>(up, left), up, left, T);
-  mux<S>(lt<S>(T, D), T, D, X);
+  mux<S>(lt<S>(left, D), left, D, T);
+  mux<S>(lt<S>(up, T), up, T, X);
   ssub_const<S, K::g, KILL>(X, kill, H);
 #pragma unroll
   for (int i = 0; i < S; ++i) Dp[i] = D[i];
