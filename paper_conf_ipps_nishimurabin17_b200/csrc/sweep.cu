@@ -59,6 +59,7 @@ __device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
+
 // Target chunk that straddles two groups of a stream (only when n % 32 != 0):
 // lane k gathers positions col.. of pair 32g+k, continuing into pair
 // 32(g+1)+k after the row end; folded H / L as tr_load_fold.  Out of line:

@@ -430,3 +430,20 @@ def test_filter_c2_full_size_sampled():
     sample = np.sort(rng.choice(P, size=4096, replace=False))
     want = oracle.sw_batch(q[sample], t[sample], 2, -1, -1) > tau
     np.testing.assert_array_equal(bits[sample].astype(bool), want)
+
+
+# ---------------------------------------------------------------- few long groups (row-skewed kernel)
+
+
+@pytest.mark.parametrize("P,m,n", [(2048, 128, 4096), (100, 100, 4000), (64, 97, 3200), (33, 128, 5000)])
+def test_few_long_groups(P, m, n):
+    """Few groups of long targets (the paper's shape, scaled down), incl.
+    padded rows, ragged n (chunks straddling groups) and ragged P."""
+    q, t = synth.gen_pairs(5150 + m + n, P, m, n, planted=True)
+    check_full(q, t)
+
+
+def test_few_long_groups_constants_and_filter():
+    q, t = synth.gen_pairs(5252, 96, 120, 3900, planted=True)
+    check_full(q, t, 3, -2, -1, 12)
+    _check_filter(q, t, 150)
