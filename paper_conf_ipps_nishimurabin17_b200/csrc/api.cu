@@ -55,7 +55,7 @@ namespace bpbc {
 namespace {
 
 SweepEntry g_table[2][kNumVariants][kNumRL][13];  // [mode][variant][rl][S - 4]
-SweepEntry g_striped[2][kNumStripeRV][3][13];     // [mode][stripe R][kind][S - 4]
+SweepEntry g_striped[2][3][13];                   // [mode][kind][S - 4]
 SweepEntry g_mw[2][kNumMw][3][13];                // [mode][(R, W)][kind][S - 4]
 SweepEntry g_planes[2][kNumVariants][2][13];      // [mode][variant][rl 0..1][S - 4]
 std::once_flag g_table_once;
@@ -113,9 +113,7 @@ Layout layout(int64_t P, int mq, int nt) {
   Layout L;
   L.G = (P + 31) / 32;
   // room for the striped / multi-warp kernels' partials: 32 lanes per 128 rows
-  // (per 64 rows when the opt-in few-groups split may use R = 2 warps)
-  const int rows_per_slot = getenv("BPBC_SPLIT_FEW_GROUPS") ? kMinStripeRows : 128;
-  L.stripes = (mq + rows_per_slot - 1) / rows_per_slot;
+  L.stripes = (mq + kStripeRows - 1) / kStripeRows;
   if (L.stripes == 3) L.stripes = 4;  // multi-warp W = 3 runs as W = 4
   // the global boundary buffer is only used by the sequential striped kernel
   const bool may_stripe = mq > 512 || (mq > 128 && getenv("BPBC_NO_MULTIWARP"));
@@ -142,7 +140,6 @@ Layout layout(int64_t P, int mq, int nt) {
 
 struct Plan {
   int circuit, consts, rl, width, cap;
-  int stripe_rv = 0;  // striped kernels: index into kStripeRV
   bool pad;
   int ops;
 };
@@ -150,7 +147,6 @@ struct Plan {
 
 // Choose the circuit, the evaluated width and the tiling.
 int make_plan(int mq, int c1, int c2, int g, int S, Plan* p) {
-  p->stripe_rv = 0;
   if (mq <= 32) p->rl = 0;
   else if (mq <= 64) p->rl = 1;
   else if (mq <= 128) p->rl = 2;
@@ -220,22 +216,11 @@ struct Dispatch {
 
 // Multi-warp variant for this plan, or -1: long queries up to
 // 512 rows (R = 4, one warp per 128 rows) and the wide-plane 129..256 case.
-int pick_mw(int mq, const Plan& p, int64_t G, int64_t short_cap) {
-  auto idx = [](int R, int W) {
-    for (int i = 0; i < kNumMw; ++i)
-      if (kMwR[i] == R && kMwW[i] == W) return i;
-    return -1;
-  };
-  if (p.rl < 0) {  // the plan wants stripes
-    if (mq <= 512) return idx(4, (mq + 127) / 128 <= 2 ? 2 : 4);  // W = 3 runs as 4
-    return -1;
-  }
-  // Few long groups (the paper's shape, G = 1024): splitting 128 rows over
-  // two R = 2 warps was measured 9 % SLOWER than one R = 4 warp per group
-  // (4 566 vs 5 016 GCUPS) -- the per-cell overhead of R = 2 outweighs the
-  // doubled warp count -- so the small-G split is only taken on request.
-  if (getenv("BPBC_SPLIT_FEW_GROUPS") && G > 0 && G * 2 <= short_cap && mq > 64 && mq <= 256)
-    return idx(2, (mq + 63) / 64 <= 2 ? 2 : 4);
+int pick_mw(int mq, const Plan& p) {
+  if (p.rl >= 0 || mq > 512) return -1;  // single-warp plan, or sequential stripes
+  const int W = (mq + 127) / 128 <= 2 ? 2 : 4;  // W = 3 runs as 4
+  for (int i = 0; i < kNumMw; ++i)
+    if (kMwR[i] == 4 && kMwW[i] == W) return i;
   return -1;
 }
 
@@ -273,8 +258,7 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int nt, int c1, int c2, int g, int S
   const Plan& plan = d->plan;
   d->striped = plan.rl < 0;
   d->ent = d->striped
-               ? g_striped[mode][plan.stripe_rv]
-                          [plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]
+               ? g_striped[mode][plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]
                           [plan.width - 4]
                : g_table[mode][variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl]
                         [plan.width - 4];
@@ -289,13 +273,13 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int nt, int c1, int c2, int g, int S
     }
   }
   if (!d->ent.launch) return BPBC_ERR_UNSUPPORTED;
-  d->R = d->striped ? kStripeRV[plan.stripe_rv] : kRLR[plan.rl];
+  d->R = d->striped ? kStripeR : kRLR[plan.rl];
   d->L = d->striped ? 32 : kRLL[plan.rl];
   int nb = occupancy_blocks(d->ent.func);
   if (nb < 0) return cuda_fail(ctx, cudaGetLastError(), "occupancy");
   if (max_blocks_env() > 0 && nb > max_blocks_env()) nb = max_blocks_env();
   d->cap_streams = int64_t(ctx->num_sms) * nb * 4 * (32 / d->L);
-  d->mw = getenv("BPBC_NO_MULTIWARP") ? -1 : pick_mw(mq, plan, G, d->cap_streams);
+  d->mw = getenv("BPBC_NO_MULTIWARP") ? -1 : pick_mw(mq, plan);
   if (d->mw >= 0) {
     const SweepEntry e =
         g_mw[mode][d->mw][plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]

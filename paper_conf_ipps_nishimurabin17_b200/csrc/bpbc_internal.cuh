@@ -52,14 +52,16 @@ struct SweepArgs {
   const uint32_t* bzero;  // 16 zero words
 };
 
-// Long queries: stripes of R rows per lane x 32 lanes, R in kStripeRV.
-constexpr int kNumStripeRV = 1;
-constexpr int kStripeRV[kNumStripeRV] = {4};  // R = 2 measured 1.7x slower at C5
-constexpr int kMinStripeRows = 64;  // workspace is sized for the smallest stripes
+// Long queries: stripes of kStripeR rows per lane x 32 lanes (R = 2 stripes
+// were measured 1.7x slower at C5).
+constexpr int kStripeR = 4;
+constexpr int kStripeRows = 32 * kStripeR;
 // Multi-warp groups (sw_sweep_mw_kernel): (R rows per lane, W warps per group)
-constexpr int kNumMw = 4;
-constexpr int kMwR[kNumMw] = {2, 2, 4, 4};
-constexpr int kMwW[kNumMw] = {2, 4, 2, 4};
+// (R = 2 variants splitting 128-row groups over two warps were measured
+// slower than one R = 4 warp and removed.)
+constexpr int kNumMw = 2;
+constexpr int kMwR[kNumMw] = {4, 4};
+constexpr int kMwW[kNumMw] = {2, 4};
 constexpr int kMaxShortRows = 256;     // m <= 256: the short kernel
 constexpr int64_t kMaxStripeStreams = 4096;
 constexpr int64_t kMaxBoundaryBytes = int64_t(1) << 30;
@@ -79,12 +81,12 @@ SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
 
 // Registration hooks, one per (score width, mode): sweep.cu is compiled once
 // per pair with -DBPBC_S=S -DBPBC_MODE=M.  tab: [variant][rl][S-4] of the
-// short kernel, stab: [stripe R variant][striped kind][S-4] (0 exact (+2,-1,-1), 1 saturating
+// short kernel, stab: [striped kind][S-4] (0 exact (+2,-1,-1), 1 saturating
 // (+2,-1,-1), 2 saturating runtime constants).
 #define BPBC_DECLARE_REG(S)                                                       \
-  void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13], \
+  void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
                                 SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]);    \
-  void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13], \
+  void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
                                 SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]);
 BPBC_DECLARE_REG(4)
 BPBC_DECLARE_REG(5)

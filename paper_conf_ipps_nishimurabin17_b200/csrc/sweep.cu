@@ -886,16 +886,16 @@ void launch_striped(const SweepArgs& a, const KRun& kr, int grid, int block, cud
   }
 }
 
-template <int S, int RV>
-void reg_striped(SweepEntry (*stab)[3][13]) {
-  constexpr int R = kStripeRV[RV];
+template <int S>
+void reg_striped(SweepEntry (*stab)[13]) {
+  constexpr int R = kStripeR;
   using K211 = KFix<2, 1, 1>;
-  stab[RV][0][S - 4] = {&launch_striped<S, kExact, K211, R>,
-                        (const void*)&sw_sweep_striped_kernel<S, kExact, K211, R>};
-  stab[RV][1][S - 4] = {&launch_striped<S, kSat, K211, R>,
-                        (const void*)&sw_sweep_striped_kernel<S, kSat, K211, R>};
-  stab[RV][2][S - 4] = {&launch_striped<S, kSat, KRun, R>,
-                        (const void*)&sw_sweep_striped_kernel<S, kSat, KRun, R>};
+  stab[0][S - 4] = {&launch_striped<S, kExact, K211, R>,
+                    (const void*)&sw_sweep_striped_kernel<S, kExact, K211, R>};
+  stab[1][S - 4] = {&launch_striped<S, kSat, K211, R>,
+                    (const void*)&sw_sweep_striped_kernel<S, kSat, K211, R>};
+  stab[2][S - 4] = {&launch_striped<S, kSat, KRun, R>,
+                    (const void*)&sw_sweep_striped_kernel<S, kSat, KRun, R>};
 }
 
 template <int S, int R, int L, int CIRC, bool PAD, class K>
@@ -942,7 +942,7 @@ void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
 #define BPBC_CAT2(a, b) a##b
 #define BPBC_CAT(a, b) BPBC_CAT2(a, b)
 #define BPBC_REGNAME BPBC_CAT(BPBC_CAT(BPBC_CAT(register_sweep_s, BPBC_S), _m), BPBC_MODE)
-void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13],
+void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],
                   SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]) {
   reg_planes<BPBC_S, 0, false>(ptab);
   reg_planes<BPBC_S, 1, false>(ptab);
@@ -950,8 +950,6 @@ void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13],
   reg_planes<BPBC_S, 1, true>(ptab);
   reg_mw<BPBC_S, 0>(mtab);
   reg_mw<BPBC_S, 1>(mtab);
-  reg_mw<BPBC_S, 2>(mtab);
-  reg_mw<BPBC_S, 3>(mtab);
   reg_rl<BPBC_S, 0, false>(tab);
   reg_rl<BPBC_S, 1, false>(tab);
   reg_rl<BPBC_S, 2, false>(tab);
@@ -960,7 +958,7 @@ void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[3][13],
   reg_rl<BPBC_S, 1, true>(tab);
   reg_rl<BPBC_S, 2, true>(tab);
   reg_rl<BPBC_S, 3, true>(tab);
-  reg_striped<BPBC_S, 0>(stab);
+  reg_striped<BPBC_S>(stab);
 }
 
 }  // namespace bpbc
