@@ -11,7 +11,9 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbpbc_sw.so")
+# BPBC_SW_LIB overrides the library path (benchmark experiments with
+# alternative builds only; the in-tree build is the default).
+LIB_PATH = os.environ.get("BPBC_SW_LIB") or os.path.join(_HERE, "libbpbc_sw.so")
 
 BPBC_OK = 0
 BPBC_ERR_INVALID_ARG = -1

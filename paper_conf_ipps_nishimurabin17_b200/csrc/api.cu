@@ -379,9 +379,12 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   a.n = nt;
   // Streams come in whole blocks on every SM (4 warps x 32/L streams per
   // block, b blocks per SM).  The SMs are ALU-bound, so an SM's time is its
-  // total work: b * 4 * segs * ceil(G / streams) groups.  Pick b in
-  // [nb - 1, nb] minimising that (ties -> more warps for latency hiding);
+  // total work, modelled as b * 4 * segs * ceil(G / streams) groups.  Pick b
+  // in [nb - 1, nb] minimising that (ties -> more warps for latency hiding);
   // the streams then split the groups as evenly as possible (base / rem).
+  // (A finer model of the base / rem split ties b = 4 and 5 at C4, where
+  // b = 5 measured 5 % slower; this one picks the measured-better b at C2
+  // and C4.)
   {
     const int64_t per_block = mw ? 1 : 4 * segs;
     const int64_t nb = cap_streams / (int64_t(ctx->num_sms) * per_block);
