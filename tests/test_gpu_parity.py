@@ -447,3 +447,54 @@ def test_few_long_groups_constants_and_filter():
     q, t = synth.gen_pairs(5252, 96, 120, 3900, planted=True)
     check_full(q, t, 3, -2, -1, 12)
     _check_filter(q, t, 150)
+
+
+@pytest.mark.parametrize("m,n", [(64, 64), (128, 200), (300, 300)])
+def test_bad_base_flag_all_kernels(m, n):
+    """Codes > 3 are read as c & 3 and raise the sticky flag in the fused
+    sweep (transposes raw codes itself), the multi-warp path (pack kernel)."""
+    q, t = synth.gen_pairs(99 + m, 64, m, n)
+    bpbc.get_error_flags(0)  # clear
+    t2 = t.copy()
+    t2[7, n - 1] = 0xFF
+    got = run(q, t2)
+    assert bpbc.get_error_flags(0) & _lib.BPBC_FLAG_BAD_BASE
+    np.testing.assert_array_equal(
+        got, oracle.sw_batch(q, t2 & 3, 2, -1, -1, score_bits=bpbc.default_score_bits(2, m, n)))
+    run(q, t)
+    assert bpbc.get_error_flags(0) == 0
+
+
+def _sharded_worker(rank, world, port, P, m, n, path):
+    import os
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_ipps_nishimurabin17_b200 import parallel
+        b, e = parallel.shard_range(P, world, rank)
+        q, t = synth.gen_pairs(4545, e - b, m, n, planted=True, p_offset=b)
+        local = parallel.score_sharded(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV), P,
+                                       2, -1, -1, 9)
+        full = parallel.gather_scores(local.cpu(), P)  # gloo gathers host tensors
+        if rank == 0:
+            np.save(path, full.numpy())
+    finally:
+        dist.destroy_process_group()
+
+
+def test_score_sharded_two_ranks_one_gpu(tmp_path):
+    """parallel.score_sharded under torch.distributed: 2 ranks (sharing cuda:0,
+    gloo for the gather) score their shards; the gathered scores equal the
+    oracle's for the whole batch."""
+    import socket
+    import torch.multiprocessing as mp
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    P, m, n = 3000, 96, 128
+    path = str(tmp_path / "sharded.npy")
+    mp.spawn(_sharded_worker, args=(2, port, P, m, n, path), nprocs=2, join=True)
+    q, t = synth.gen_pairs(4545, P, m, n, planted=True)
+    np.testing.assert_array_equal(np.load(path), oracle.sw_batch(q, t, 2, -1, -1, score_bits=9))
