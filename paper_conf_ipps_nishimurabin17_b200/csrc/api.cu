@@ -446,8 +446,9 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
                              o.scratch, o.scratch_bytes, ctx->num_sms, st);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "filter epilogue");
   } else {
-    e = launch_extract(Mpart, lay.G, L * a.stripes * W, plan.width, P, plan.cap, o.scores,
-                       ctx->num_sms, st);
+    // the exact circuit's partial maxima carry the offset g (finish_exact)
+    e = launch_extract(Mpart, lay.G, L * a.stripes * W, plan.width, P,
+                       plan.circuit == kExact ? g : 0, plan.cap, o.scores, ctx->num_sms, st);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "extract");
   }
   if (ev[3]) cudaEventRecord(ev[3], st);
@@ -834,7 +835,7 @@ int bpbc_sw_untranspose(bpbc_sw_ctx* ctx, const uint32_t* partial, int64_t num_g
   if (num_groups == 0 || num_pairs == 0) return BPBC_OK;
   if (!partial || !out) return BPBC_ERR_INVALID_ARG;
   DeviceGuard dg(ctx->device);
-  cudaError_t e = launch_extract(partial, num_groups, lanes, s, num_pairs, cap, out,
+  cudaError_t e = launch_extract(partial, num_groups, lanes, s, num_pairs, 0, cap, out,
                                  ctx->num_sms, static_cast<cudaStream_t>(stream));
   return e == cudaSuccess ? BPBC_OK : cuda_fail(ctx, e, "untranspose");
 }

@@ -123,8 +123,9 @@ cudaError_t launch_wordwise(const uint8_t* q, const uint8_t* t, int64_t P, int m
                             int c1, int c2, int g, int32_t* out, void* ws, int num_sms,
                             cudaStream_t st);
 // extract.cu
+// score = min(max(untransposed max - offset, 0), cap)
 cudaError_t launch_extract(const uint32_t* partial, int64_t num_groups, int lanes, int s,
-                           int64_t num_pairs, int32_t cap, int32_t* out, int num_sms,
-                           cudaStream_t stream);
+                           int64_t num_pairs, int32_t offset, int32_t cap, int32_t* out,
+                           int num_sms, cudaStream_t stream);
 
 }  // namespace bpbc

@@ -248,9 +248,11 @@ BPBC_HD void cell_exact(const uint32_t (&up)[S], const uint32_t (&left)[S],
 // up - g or left - g, that neighbour would hold H* + g > H*.  Every D <= H.
 // Hence max_ij H = max(0, max_ij D) with D = diag + w (saturating cell), and
 // max_ij H = max(0, max_ij D' - g) with D' = diag + w + g (exact cell).  The
-// lane keeps M over D (2S LOP3 per cell, as over H) and the exact kernel
-// subtracts g once per group (finish_exact).  D is ready long before H, so
-// the M chain runs beside the comparator chain instead of after it.
+// lane keeps M over D (2S LOP3 per cell, as over H); for the exact circuit
+// the sweep stores max D' and extract.cu subtracts g from the untransposed
+// integer once per pair (finish_exact is the bit-sliced form of that step,
+// used by the host circuit tests).  D is ready long before H, so the M chain
+// runs beside the comparator chain instead of after it.
 template <int S, int G>
 BPBC_HD void finish_exact(const uint32_t (&Mp)[S], uint32_t (&M)[S]) {
   ssub_const<S, G, false>(Mp, 0u, M);

@@ -199,27 +199,23 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   int64_t gi = -1;   // my current group within the stream
   uint32_t flag = 0; // threshold mode: pairs with a cell > tau so far
 
-  // One wavefront step with target planes y of my current column.
-  auto step = [&](const uint2 y) {
+  // One wavefront step with target planes y of my current column.  SW: the
+  // step may be a lane's group switch (the warp runs phases in which no lane
+  // switches without the per-step check).
+  auto step = [&](const uint2 y, auto SW) {
     uint32_t up[S];
 #pragma unroll
     for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
 
-    if (cnt == 0) {  // column 0 of my next group (divergent, once per group)
+    if (decltype(SW)::value && cnt == 0) {  // column 0 of my next group (divergent, once per group)
       if (gi >= 0 && gi < Gs) {
         if constexpr (BPBC_MODE == kModeThreshold) {
           a.Mpart[(gb + gi) * L + sl] = flag;  // one flag word per lane
         } else {
           uint32_t* dst = a.Mpart + ((gb + gi) * L + sl) * S;
-          if constexpr (CIRC == kExact) {
-            uint32_t F[S];
-            finish_exact<S, K::g>(M, F);  // M tracked D' = diag + w + g
+          // exact circuit: M tracked D' = diag + w + g; extract subtracts g
 #pragma unroll
-            for (int i = 0; i < S; ++i) dst[i] = F[i];
-          } else {
-#pragma unroll
-            for (int i = 0; i < S; ++i) dst[i] = M[i];
-          }
+          for (int i = 0; i < S; ++i) dst[i] = M[i];
         }
       }
       ++gi;
@@ -239,7 +235,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
       }
       cnt = a.n;
     }
-    --cnt;
+    if (decltype(SW)::value) --cnt;
 
     uint32_t dg[S], u[S];
 #pragma unroll
@@ -305,11 +301,25 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     }
     __syncwarp();
     const uint2* yb = &yr[seg][(32 * p - sl) & 127];  // my 32 columns of this phase
+    // a lane switches groups in this phase iff its countdown is below 32.
+    // Two copies of the loop body must fit the instruction cache together
+    // (4 warps per SMSP run both): at R = 8 one copy is ~27 KB and two copies
+    // measured 16 % slower (C3), so R = 8 keeps only the checked loop.
+    if (R > 4 || __any_sync(0xFFFFFFFFu, cnt < 32)) {
 #pragma unroll 1
-    for (int i = 0; i < 32; i += 2) {
-      const uint2 y0 = yb[i], y1 = yb[i + 1];
-      step(y0);
-      step(y1);
+      for (int i = 0; i < 32; i += 2) {
+        const uint2 y0 = yb[i], y1 = yb[i + 1];
+        step(y0, std::true_type{});
+        step(y1, std::true_type{});
+      }
+    } else {
+#pragma unroll 1
+      for (int i = 0; i < 32; i += 2) {
+        const uint2 y0 = yb[i], y1 = yb[i + 1];
+        step(y0, std::false_type{});
+        step(y1, std::false_type{});
+      }
+      cnt -= 32;
     }
   }
   if (__any_sync(0xFFFFFFFFu, bad != 0) && lane == 0) atomicOr(a.flags, BPBC_FLAG_BAD_BASE);
@@ -388,15 +398,9 @@ __global__ void __launch_bounds__(128) sw_sweep_planes_kernel(const SweepArgs a,
           a.Mpart[(gb + gi) * L + sl] = flag;  // one flag word per lane
         } else {
           uint32_t* dst = a.Mpart + ((gb + gi) * L + sl) * S;
-          if constexpr (CIRC == kExact) {
-            uint32_t F[S];
-            finish_exact<S, K::g>(M, F);  // M tracked D' = diag + w + g
+          // exact circuit: M tracked D' = diag + w + g; extract subtracts g
 #pragma unroll
-            for (int i = 0; i < S; ++i) dst[i] = F[i];
-          } else {
-#pragma unroll
-            for (int i = 0; i < S; ++i) dst[i] = M[i];
-          }
+          for (int i = 0; i < S; ++i) dst[i] = M[i];
         }
       }
       ++gi;
@@ -551,15 +555,9 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
           a.Mpart[(g * stripes + kk) * L + sl] = flag;
         } else {
           uint32_t* dst = a.Mpart + ((g * stripes + kk) * L + sl) * S;
-          if constexpr (CIRC == kExact) {
-            uint32_t F[S];
-            finish_exact<S, K::g>(M, F);
+          // exact circuit: M tracked D' = diag + w + g; extract subtracts g
 #pragma unroll
-            for (int i = 0; i < S; ++i) dst[i] = F[i];
-          } else {
-#pragma unroll
-            for (int i = 0; i < S; ++i) dst[i] = M[i];
-          }
+          for (int i = 0; i < S; ++i) dst[i] = M[i];
         }
       }
       ++vi;
@@ -740,7 +738,7 @@ __global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_m
   int64_t gi = -1;
   uint32_t flag = 0;
 
-  auto step = [&](const uint2 y) {
+  auto step = [&](const uint2 y, auto SW) {  // SW: as in sw_sweep_kernel
     uint32_t up[S];
     {
       const uint4* b4 = reinterpret_cast<const uint4*>(rbase + (off & rmask));
@@ -754,21 +752,15 @@ __global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_m
             up[4 * q + e] = mad_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][4 * q + e], 1), nz, w[e]);
       }
     }
-    if (cnt == 0) {  // column 0 of my next group (divergent, once per group)
+    if (decltype(SW)::value && cnt == 0) {  // column 0 of my next group (divergent, once per group)
       if (gi >= 0 && gi < Gs) {
         if constexpr (BPBC_MODE == kModeThreshold) {
           a.Mpart[((gb + gi) * W + wk) * 32 + lane] = flag;
         } else {
           uint32_t* dst = a.Mpart + (((gb + gi) * W + wk) * 32 + lane) * S;
-          if constexpr (CIRC == kExact) {
-            uint32_t F[S];
-            finish_exact<S, K::g>(M, F);
+          // exact circuit: M tracked D' = diag + w + g; extract subtracts g
 #pragma unroll
-            for (int i = 0; i < S; ++i) dst[i] = F[i];
-          } else {
-#pragma unroll
-            for (int i = 0; i < S; ++i) dst[i] = M[i];
-          }
+          for (int i = 0; i < S; ++i) dst[i] = M[i];
         }
       }
       ++gi;
@@ -790,7 +782,7 @@ __global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_m
       fetch_x(gi + 1, int((gi + 1) & 1));
       cnt = a.n;
     }
-    --cnt;
+    if (decltype(SW)::value) --cnt;
     uint32_t dg[S], u[S];
 #pragma unroll
     for (int i = 0; i < S; ++i) {
@@ -836,12 +828,23 @@ __global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_m
 
   uint2 y0 = __ldg(yp), y1;
   for (int64_t tau = 0; tau < a.steps; tau += 32) {
+    if (__any_sync(0xFFFFFFFFu, cnt < 32)) {  // a lane of this warp switches groups
 #pragma unroll 1
-    for (int i = 0; i < 32; i += 2) {
-      y1 = __ldg(yp + tau + i + 1);
-      step(y0);
-      y0 = __ldg(yp + tau + i + 2);
-      step(y1);
+      for (int i = 0; i < 32; i += 2) {
+        y1 = __ldg(yp + tau + i + 1);
+        step(y0, std::true_type{});
+        y0 = __ldg(yp + tau + i + 2);
+        step(y1, std::true_type{});
+      }
+    } else {
+#pragma unroll 1
+      for (int i = 0; i < 32; i += 2) {
+        y1 = __ldg(yp + tau + i + 1);
+        step(y0, std::false_type{});
+        y0 = __ldg(yp + tau + i + 2);
+        step(y1, std::false_type{});
+      }
+      cnt -= 32;
     }
     __syncthreads();  // phase boundary: ring writes of this phase -> reads of the next
   }
