@@ -131,6 +131,10 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   int64_t Gs, gb;
   seg_range(seg, gb, Gs);
   const uint32_t nz = opaque(sl != 0 ? 1u : 0u);
+  // multiplier 0 for the state reset at a group switch: the reset runs as
+  // IMADs on the FMA pipe instead of register-pair clears on the ALU pipe,
+  // which the cell circuits saturate
+  const uint32_t z0 = opaque(uint32_t(a.m) >> 31);  // 0 (m > 0), unknown to ptxas
   uint32_t kill[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) kill[r] = PAD ? opaque((sl * R + r >= a.m) ? 0xFFFFFFFFu : 0u) : 0u;
@@ -196,8 +200,13 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
 #pragma unroll
   for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
   int cnt = sl;      // steps until my next group starts (J % n == 0)
-  int64_t gi = -1;   // my current group within the stream
+  int gi = -1;       // my current group within the stream
   uint32_t flag = 0; // threshold mode: pairs with a cell > tau so far
+  const int gsn = int(Gs);  // groups of my stream (< 2^31: P < 2^36)
+  // my partial-max slot of the current group, advanced at every switch
+  constexpr int kMW = BPBC_MODE == kModeThreshold ? L : L * S;
+  uint32_t* mdst = a.Mpart + (gb * L + sl) * (kMW / L);
+  const uint2* xrow = &xr[0][lane][0];  // + slot * 32 * R
 
   // One wavefront step with target planes y of my current column.  SW: the
   // step may be a lane's group switch (the warp runs phases in which no lane
@@ -208,28 +217,29 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
 
     if (decltype(SW)::value && cnt == 0) {  // column 0 of my next group (divergent, once per group)
-      if (gi >= 0 && gi < Gs) {
+      if (gi >= 0 && gi < gsn) {
         if constexpr (BPBC_MODE == kModeThreshold) {
-          a.Mpart[(gb + gi) * L + sl] = flag;  // one flag word per lane
+          *mdst = flag;  // one flag word per lane
         } else {
-          uint32_t* dst = a.Mpart + ((gb + gi) * L + sl) * S;
           // exact circuit: M tracked D' = diag + w + g; extract subtracts g
 #pragma unroll
-          for (int i = 0; i < S; ++i) dst[i] = M[i];
+          for (int i = 0; i < S; ++i) mdst[i] = M[i];
         }
+        mdst += kMW;
       }
       ++gi;
-      flag = 0;
+      flag = mul_lo(flag, z0);
 #pragma unroll
       for (int i = 0; i < S; ++i) {
-        M[i] = 0;
-        dtop[i] = 0;
+        M[i] = mul_lo(M[i], z0);
+        dtop[i] = mul_lo(dtop[i], z0);
 #pragma unroll
-        for (int r = 0; r < R; ++r) H[r][i] = 0;
+        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], z0);
       }
+      const uint2* xv = xrow + (gi & 1) * (32 * R);
 #pragma unroll
       for (int r = 0; r < R; ++r) {
-        const uint2 v = xr[int(gi & 1)][lane][r];
+        const uint2 v = xv[r];
         xh[r] = v.x;
         xl[r] = v.y;
       }
@@ -698,6 +708,7 @@ __global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_m
   __syncthreads();
 
   const uint32_t nz = opaque(lane != 0 ? 1u : 0u);
+  const uint32_t z0 = opaque(uint32_t(a.m) >> 31);  // 0: state reset on the FMA pipe
   const int row0 = wk * LR + lane * R;
   uint32_t kill[R];
 #pragma unroll
@@ -764,13 +775,13 @@ __global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_m
         }
       }
       ++gi;
-      flag = 0;
+      flag = mul_lo(flag, z0);
 #pragma unroll
       for (int i = 0; i < S; ++i) {
-        M[i] = 0;
-        dtop[i] = 0;
+        M[i] = mul_lo(M[i], z0);
+        dtop[i] = mul_lo(dtop[i], z0);
 #pragma unroll
-        for (int r = 0; r < R; ++r) H[r][i] = 0;
+        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], z0);
       }
       cp_async_wait_all();
 #pragma unroll
