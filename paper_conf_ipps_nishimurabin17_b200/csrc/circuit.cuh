@@ -163,28 +163,41 @@ BPBC_HD uint32_t mismatch_flag(uint32_t xh, uint32_t xl, uint32_t yh, uint32_t y
 
 // U = max(X - G, 0) for a compile-time G, forced to 0 where kill = 1.
 // Borrow chain b_{i+1} = MAJ(~X_i, G_i, b_i), output U_i = (X_i^G_i^b_i) & ~b_S.
-// 2S LOP3 (one less when G_0 = 0 ... folded by ptxas).
+// 2S - 1 LOP3 (G_0 = 0: b_1 = 0 is constant-folded by ptxas; G_0 = 1: see below).
+//
+// When G_0 = 1 the first borrow is b_1 = ~X_0: it is never materialised;
+// its two consumers (b_2 and U_1) read X_0 with the inversion folded into
+// their truth tables, which saves one gate (2S - 1 in total).
 template <int S, int G, bool KILL>
 BPBC_HD void ssub_const(const uint32_t (&X)[S], uint32_t kill, uint32_t (&U)[S]) {
+  static_assert(S >= 3, "ssub_const needs S >= 3");
+  constexpr bool kB1 = (G & 1) != 0;  // b_1 = ~X_0 (virtual)
   uint32_t b[S + 1];
   b[0] = 0u;
+  b[1] = 0u;  // (unused when kB1)
   static_for<S>([&](auto I) {
     constexpr int i = decltype(I)::value;
     constexpr uint32_t g = (G >> i) & 1 ? 0xFFu : 0u;
-    if constexpr (i == S - 1 && KILL) {
+    // borrow input b_i as seen by this gate: TB, or ~TB when it is X_0
+    constexpr uint32_t bin = (kB1 && i == 1) ? (~TB & 0xFFu) : TB;
+    constexpr uint32_t maj = (~TA & g) | (~TA & bin) | (g & bin);
+    if constexpr (kB1 && i == 0) {
+      // b_1 = ~X_0: folded into the consumers
+    } else if constexpr (i == S - 1 && KILL) {
       // borrow out OR kill, still one gate: inputs (X_i, b_i, kill)
-      constexpr uint8_t t = T8((((~TA & g) | (~TA & TB) | (g & TB)) & 0xFF) | TC);
-      b[i + 1] = lop3<t>(X[i], b[i], kill);
+      constexpr uint8_t t = T8((maj & 0xFF) | TC);
+      b[i + 1] = lop3<t>(X[i], (kB1 && i == 1) ? X[0] : b[i], kill);
     } else {
-      constexpr uint8_t t = T8((~TA & g) | (~TA & TB) | (g & TB));
-      b[i + 1] = lop3<t>(X[i], b[i], 0u);
+      constexpr uint8_t t = T8(maj);
+      b[i + 1] = lop3<t>(X[i], (kB1 && i == 1) ? X[0] : b[i], 0u);
     }
   });
   static_for<S>([&](auto I) {
     constexpr int i = decltype(I)::value;
     constexpr uint32_t g = (G >> i) & 1 ? 0xFFu : 0u;
-    constexpr uint8_t t = T8((TA ^ g ^ TB) & ~TC);  // (X_i ^ G_i ^ b_i) & ~b_S
-    U[i] = lop3<t>(X[i], b[i], b[S]);
+    constexpr uint32_t bin = (kB1 && i == 1) ? (~TB & 0xFFu) : TB;
+    constexpr uint8_t t = T8((TA ^ g ^ bin) & ~TC);  // (X_i ^ G_i ^ b_i) & ~b_S
+    U[i] = lop3<t>(X[i], (kB1 && i == 1) ? X[0] : b[i], b[S]);
   });
 }
 
