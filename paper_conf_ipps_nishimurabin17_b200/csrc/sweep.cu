@@ -22,8 +22,9 @@
 //     groups back to back as one virtual target of length Gs*n, so the
 //     pipeline fill/drain (L-1 steps, the paper's (m-1)/(n+m-1) idle share)
 //     is paid once per stream, not per group;
-//   * the group switch of a lane (its column J hits a multiple of n) resets
-//     its state in a short divergent branch taken once per group per lane;
+//   * the group switch of a lane (its column J hits a multiple of n) stores
+//     its partial max and resets its state, branch-free (predicated) in the
+//     phases that contain switches;
 //   * the cell is a fixed LOP3 circuit (circuit.cuh): no branch on data.
 #include "bpbc_internal.cuh"
 #include "transpose.cuh"
@@ -48,6 +49,35 @@ __device__ __forceinline__ uint32_t mul_lo(uint32_t a, uint32_t b) {
   asm("mul.lo.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
   return r;
 }
+__device__ __forceinline__ uint32_t mul_hi(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm("mul.hi.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+
+// Predicated global store / shared load (the predicate is pr != 0): forced
+// into PTX predication so the group switch of kSwPred adds no branch.
+__device__ __forceinline__ void st_if(uint32_t* p, uint32_t v, uint32_t pr) {
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q st.global.u32 [%0], %1; }" ::"l"(p), "r"(v),
+               "r"(pr)
+               : "memory");
+}
+__device__ __forceinline__ void lds2_if(const uint2* p, uint32_t& x, uint32_t& y, uint32_t pr) {
+  const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(p));
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %3, 0; @q ld.shared.v2.u32 {%0, %1}, [%2]; }"
+               : "+r"(x), "+r"(y)
+               : "r"(s), "r"(pr)
+               : "memory");
+}
+
+// Group-switch handling of a step (sw_sweep_kernel): none in the phase, a
+// divergent branch, or branch-free predication.
+enum : int { kSwNone = 0, kSwBranch = 1, kSwPred = 2 };
+#ifndef BPBC_SWMODE
+#define BPBC_SWMODE kSwPred
+#endif
+template <int V>
+using SwMode = std::integral_constant<int, V>;
 
 // Asynchronous 8-byte global -> shared copies (cp.async, no register
 // staging): the next group's query planes are fetched while the current
@@ -210,13 +240,45 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
 
   // One wavefront step with target planes y of my current column.  SW: the
   // step may be a lane's group switch (the warp runs phases in which no lane
-  // switches without the per-step check).
+  // switches without the per-step check): kSwBranch takes the switch in a
+  // divergent branch, kSwPred runs it branch-free in every lane (predicated
+  // stores and loads, state reset by a multiply with 0/1 on the FMA pipe), so
+  // the two steps of an iteration stay one basic block the scheduler can
+  // interleave.
   auto step = [&](const uint2 y, auto SW) {
     uint32_t up[S];
 #pragma unroll
     for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
 
-    if (decltype(SW)::value && cnt == 0) {  // column 0 of my next group (divergent, once per group)
+    if constexpr (decltype(SW)::value == kSwPred) {
+      // keep = 0 at column 0 of my next group, else 1: the carry of
+      // cnt + (2^31 - 1) into bit 31, taken as mul.hi so it stays on the FMA
+      // pipe and ptxas cannot turn the resets below into selects
+      const uint32_t keep = mul_hi(uint32_t(cnt) + 0x7FFFFFFFu, 2u);
+      const bool sw = cnt == 0;
+      const uint32_t st = (sw && unsigned(gi) < unsigned(gsn)) ? 1u : 0u;
+      if constexpr (BPBC_MODE == kModeThreshold) {
+        st_if(mdst, flag, st);
+      } else {
+#pragma unroll
+        for (int i = 0; i < S; ++i) st_if(mdst + i, M[i], st);
+      }
+      mdst += st * kMW;
+      gi += sw ? 1 : 0;
+      flag = mul_lo(flag, keep);
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        M[i] = mul_lo(M[i], keep);
+        dtop[i] = mul_lo(dtop[i], keep);
+#pragma unroll
+        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], keep);
+      }
+      const uint2* xv = xrow + (gi & 1) * (32 * R);
+#pragma unroll
+      for (int r = 0; r < R; ++r) lds2_if(xv + r, xh[r], xl[r], sw ? 1u : 0u);
+      cnt = (sw ? a.n : cnt) - 1;
+    }
+    if (decltype(SW)::value == kSwBranch && cnt == 0) {  // column 0 of my next group (divergent, once per group)
       if (gi >= 0 && gi < gsn) {
         if constexpr (BPBC_MODE == kModeThreshold) {
           *mdst = flag;  // one flag word per lane
@@ -245,7 +307,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
       }
       cnt = a.n;
     }
-    if (decltype(SW)::value) --cnt;
+    if (decltype(SW)::value == kSwBranch) --cnt;
 
     uint32_t dg[S], u[S];
 #pragma unroll
@@ -315,19 +377,23 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     // Two copies of the loop body must fit the instruction cache together
     // (4 warps per SMSP run both): at R = 8 one copy is ~27 KB and two copies
     // measured 16 % slower (C3), so R = 8 keeps only the checked loop.
+    // Switch phases run branch-free (kSwPred: C2 5 743 vs 5 643 GCUPS with the
+    // divergent branch); the single R = 8 loop runs in every phase and keeps
+    // the branch (kSwPred there costs every step: C3 5 194 vs 5 429).
+    constexpr int kSw = R > 4 ? kSwBranch : BPBC_SWMODE;
     if (R > 4 || __any_sync(0xFFFFFFFFu, cnt < 32)) {
 #pragma unroll 1
       for (int i = 0; i < 32; i += 2) {
         const uint2 y0 = yb[i], y1 = yb[i + 1];
-        step(y0, std::true_type{});
-        step(y1, std::true_type{});
+        step(y0, SwMode<kSw>{});
+        step(y1, SwMode<kSw>{});
       }
     } else {
 #pragma unroll 1
       for (int i = 0; i < 32; i += 2) {
         const uint2 y0 = yb[i], y1 = yb[i + 1];
-        step(y0, std::false_type{});
-        step(y1, std::false_type{});
+        step(y0, SwMode<kSwNone>{});
+        step(y1, SwMode<kSwNone>{});
       }
       cnt -= 32;
     }
