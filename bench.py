@@ -9,7 +9,7 @@ batch of synthetic pairs already resident in HBM.  Default workload (N=1) is
 BASELINE.json configs[1] = C2: 2^20 DNA pairs, m = n = 128, +2/-1/-1, 9-bit
 slices.  For N > 1 (torchrun, one process per GPU) every rank scores its own
 C2-sized shard (weak scaling, no collective on the data path); the int32
-scores are all-gathered once after the timed region for the parity sample.
+scores are all-gathered once after the timed region.
 
 Prints ONE JSON line on rank 0 (contract in the task statement / DESIGN.md
 "Measurement"): metric, value (GCUPS, all ranks), e2e (same metric through
@@ -17,7 +17,8 @@ the host-buffer C call bpbc_sw_score_batch_host with pinned host inputs,
 H2D + D2H inside the timed region), roofline (the sweep kernel against the
 integer-logic pipe peak), cpu_baseline (the oracle on a bounded sample on
 this host's cores), clocks (nvidia-smi sampled during the timed region),
-gpu_launches, parity (a sample of pairs checked against the oracle).
+gpu_launches, parity (the GPU scores of the cpu_baseline sample checked
+against the oracle's; N=1 only, like cpu_baseline).
 
 --impl reference times the CPU oracle (oracle/) on the same config -- the
 reference arm of this tier (no reference implementation exists).
@@ -125,26 +126,31 @@ class ClockSampler:
 
 
 def cpu_baseline(cfg, target_seconds=12.0):
-    """The oracle as it stands, on a bounded sample of the workload, all host cores."""
+    """The oracle as it stands, on a bounded sample of the workload (its first
+    pairs), all host cores.  Returns the cpu_baseline object and the oracle's
+    scores of the sample, which the caller compares with the GPU's (parity)."""
     import oracle
     import synth
     threads = os.cpu_count() or 1
     m, n = cfg["m"], cfg["n"]
     seed = synth.seed_for_config(cfg["id"])
-    cal = max(threads, 256)
+    # calibrate the rate on a warm library with enough pairs per thread that
+    # thread start-up does not dominate, then size the sample to ~target_seconds
+    cal = int(min(cfg["P"], max(64 * threads, 4096)))
     q, t = synth.gen_pairs(seed, cal, m, n)
+    oracle.sw_batch(q[:threads], t[:threads], *CONSTS, score_bits=cfg["s"], threads=threads)
     t0 = time.perf_counter()
     oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
     rate = cal / max(time.perf_counter() - t0, 1e-6)
-    sample = int(min(cfg["P"], max(threads, rate * target_seconds)))
+    sample = int(min(cfg["P"], max(cal, rate * target_seconds)))
     q, t = synth.gen_pairs(seed, sample, m, n)
     t0 = time.perf_counter()
-    oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
+    want = oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
     dt = time.perf_counter() - t0
     return {"value": round(sample * m * n / dt / 1e9, 4), "unit": "GCUPS", "cores": threads,
             "kind": "oracle",
             "sample": f"first {sample} of the {cfg['P']} pairs of C{cfg['id']} "
-                      f"(m={m}, n={n}), {dt:.1f} s, scalar int32 DP, {threads} threads"}
+                      f"(m={m}, n={n}), {dt:.1f} s, scalar int32 DP, {threads} threads"}, want
 
 
 def run_reference(args, cfg):
@@ -158,8 +164,9 @@ def run_reference(args, cfg):
     m, n = cfg["m"], cfg["n"]
     seed = synth.seed_for_config(cfg["id"])
     # size one step so the whole run stays within ~1-2 minutes
-    cal = max(threads, 256)
+    cal = int(min(cfg["P"], max(64 * threads, 4096)))
     q, t = synth.gen_pairs(seed, cal, m, n)
+    oracle.sw_batch(q[:threads], t[:threads], *CONSTS, score_bits=cfg["s"], threads=threads)
     t0 = time.perf_counter()
     oracle.sw_batch(q, t, *CONSTS, score_bits=cfg["s"], threads=threads)
     rate = cal / max(time.perf_counter() - t0, 1e-6)
@@ -412,7 +419,7 @@ def main():
                        "timing": "host wall clock around bpbc_sw_score_batch_host_packed2 "
                                  "(pinned, 2-bit packed bases)"}
 
-    # ---------------- result gather (outside the timed region) + parity sample
+    # ---------------- result gather (outside the timed region)
     if world > 1:  # rank r holds the pairs of shard_range(P_total, world, r)
         full = parallel.gather_scores(out.to(cdev), P_total)
         got_all = full.cpu().numpy()
@@ -421,20 +428,6 @@ def main():
     if rank != 0:
         dist.destroy_process_group()
         return
-    import oracle
-    rng = np.random.default_rng(seed)
-    total = P_total
-    nsamp = int(min(total, 2048, max(16, 2e9 // (m * n))))  # ~2e9 oracle cells at most
-    idx = np.unique(np.concatenate([rng.choice(total, size=nsamp, replace=False),
-                                    [0, total - 1]]))
-    sq = np.empty((idx.size, m), dtype=np.uint8)
-    st_ = np.empty((idx.size, n), dtype=np.uint8)
-    for j, p in enumerate(idx):  # regenerate the sampled pairs by global index
-        synth.gen_pairs(seed, 1, m, n, p_offset=int(p), out_q=sq[j:j + 1], out_t=st_[j:j + 1],
-                        threads=1)
-    want = oracle.sw_batch(sq, st_, *CONSTS, score_bits=s)
-    parity = {"sampled_pairs": int(idx.size), "mismatches": int((got_all[idx] != want).sum()),
-              "ranks_gathered": world}
 
     # ---------------- roofline of the sweep kernel (integer-logic pipe)
     calls = max(1, phases["calls"])
@@ -465,8 +458,17 @@ def main():
                 "phase_ms_per_step": {k: round(v / calls, 4) for k, v in phases.items()
                                       if k.endswith("_ms")}}
     cpu = None
+    parity = None
     if not args.no_cpu_baseline and world == 1:
-        cpu = cpu_baseline(cfg)
+        # the cpu_baseline leg's oracle scores of the first pairs double as the
+        # bench's bit-exact parity check of the GPU results for those pairs
+        cpu, want = cpu_baseline(cfg)
+        parity = {"pairs_checked": int(want.size),
+                  "mismatches": int((got_all[:want.size] != want).sum()),
+                  "what": "GPU scores of the cpu_baseline sample vs the oracle's"}
+    # score distribution of the batch (C5: the share capped at 2^s - 1, R3)
+    scores = {"mean": round(float(got_all.mean()), 3), "max": int(got_all.max()),
+              "saturated_frac": round(float((got_all == (1 << s) - 1).mean()), 6)}
 
     line = {"metric": METRIC, "value": round(gcups, 2), "unit": "GCUPS", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup,
@@ -484,7 +486,8 @@ def main():
             "e2e": e2e, "e2e_packed2": e2e_packed2, "filter": filt, "wordwise": wordwise, "roofline": roofline, "cpu_baseline": cpu, "clocks": clocks,
             # ours per step and rank, from the library (fused sweep + extract,
             # or pack + sweep + extract)
-            "gpu_launches": plan["kernels"] * args.steps * world, "parity": parity}
+            "gpu_launches": plan["kernels"] * args.steps * world, "parity": parity,
+            "scores": scores}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
