@@ -265,7 +265,11 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int nt, int c1, int c2, int g, int S
   // single-warp plans: the fused kernel unless the target is too short for
   // its phase-granular query transposes (n < L + 32, only for L = 16)
   if (!d->striped) {
-    d->fused = nt >= kRLL[plan.rl] + 32;
+    // (a query build per group must fall on a phase start between "every
+    // lane entered the previous group" and "lane 0 needs it": some multiple
+    // of 32 in [(h-1) n + L, h n] -- always when n >= L + 31, and at h n
+    // itself when n is a multiple of 32)
+    d->fused = nt >= kRLL[plan.rl] + 32 || nt % 32 == 0;
     if (!d->fused) {
       if (plan.rl > 1) return BPBC_ERR_UNSUPPORTED;  // (cannot happen: n >= m > 64)
       d->ent = g_planes[mode][variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl]
