@@ -101,6 +101,24 @@ def test_lengths(m, n):
     check_full(q, t)
 
 
+@pytest.mark.parametrize("m,n", [(32, 32), (7, 32), (32, 7), (31, 64), (16, 96), (20, 40)])
+@pytest.mark.parametrize("packed2", [False, True])
+def test_short_targets_fused(m, n, packed2):
+    """Targets shorter than L + 32 whose length is a multiple of 32 take the
+    fused kernel (one query build per phase, at the group boundary itself);
+    others (n = 40 < 48) the planes kernel.  Both inputs formats."""
+    q, t = synth.gen_pairs(5400 + m * 7 + n, 300, m, n, planted=True)
+    want = oracle.sw_batch(q, t, 2, -1, -1)
+    if packed2:
+        dq = torch.from_numpy(synth.pack2bit(q)).to(DEV)
+        dt = torch.from_numpy(synth.pack2bit(t)).to(DEV)
+        got = bpbc.score_batch_packed2(dq, dt, m, n, 2, -1, -1).cpu().numpy()
+    else:
+        got = run(q, t)
+    np.testing.assert_array_equal(got, want)
+    assert bpbc.last_plan(0)["fused"] == (max(m, n) % 32 == 0)
+
+
 @pytest.mark.parametrize("s", list(range(4, 17)))
 def test_every_width_spec_consts(s):
     q, t = synth.gen_pairs(600 + s, 512, 48, 80, planted=True)
