@@ -457,6 +457,27 @@ def main():
                               f"{sm_max:.0f} MHz (B300_MICROARCH alu rt=2/SMSP)",
                 "phase_ms_per_step": {k: round(v / calls, 4) for k, v in phases.items()
                                       if k.endswith("_ms")}}
+    # W2B (pack_kernel) against the measured HBM copy bandwidth, when the plan
+    # runs it (multi-warp, striped and short-target plans); the fused sweep
+    # transposes the raw codes itself and has no W2B launch
+    w2b = None
+    w2b_ms = phases.get("w2b_ms", 0.0) / calls
+    if not plan.get("fused") and w2b_ms > 0:
+        hbm = 6552.0
+        try:
+            hbm = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
+            hbm_src = "MEASURED_PEAKS.json hbm_gbs"
+        except Exception:
+            hbm_src = "fallback 6552 GB/s (MEASURED_PEAKS.json unreadable)"
+        mq, nt = min(m, n), max(m, n)
+        groups = (P + 31) // 32
+        nbytes = P * (m + n) + 8 * groups * (mq + nt)  # u8 codes read + uint2 planes written
+        gbs = nbytes / (w2b_ms / 1e3) / 1e9
+        w2b = {"bound": "hbm", "kernel": "pack_kernel", "achieved": round(gbs, 1),
+               "peak": hbm, "unit": "GB/s", "frac": round(gbs / hbm, 4),
+               "bytes_per_launch": nbytes, "ms_per_launch": round(w2b_ms, 4),
+               "peak_source": hbm_src}
+
     cpu = None
     parity = None
     if not args.no_cpu_baseline and world == 1:
@@ -487,7 +508,7 @@ def main():
             # ours per step and rank, from the library (fused sweep + extract,
             # or pack + sweep + extract)
             "gpu_launches": plan["kernels"] * args.steps * world, "parity": parity,
-            "scores": scores}
+            "scores": scores, "w2b_roofline": w2b}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
