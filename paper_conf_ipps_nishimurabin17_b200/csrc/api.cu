@@ -218,7 +218,7 @@ struct Dispatch {
 // 512 rows (R = 4, one warp per 128 rows) and the wide-plane 129..256 case.
 int pick_mw(int mq, const Plan& p) {
   if (p.rl >= 0 || mq > 512) return -1;  // single-warp plan, or sequential stripes
-  const int W = (mq + 127) / 128 <= 2 ? 2 : 4;  // W = 3 runs as 4
+  const int W = (mq + 127) / 128 <= 2 ? 2 : 4;  // W = 3 runs as 4 (bpbc_internal.cuh)
   for (int i = 0; i < kNumMw; ++i)
     if (kMwR[i] == 4 && kMwW[i] == W) return i;
   return -1;
@@ -296,11 +296,12 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int nt, int c1, int c2, int g, int S
       d->W = kMwW[d->mw];
       d->L = 32;
       int nbm = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nbm, e.func, 32 * d->W, 0) !=
+      const int gpb = mw_groups_per_block(d->W);
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nbm, e.func, 32 * d->W * gpb, 0) !=
           cudaSuccess)
         return cuda_fail(ctx, cudaGetLastError(), "occupancy");
       if (nbm < 1) nbm = 1;
-      d->cap_streams = int64_t(ctx->num_sms) * nbm;  // one stream per block
+      d->cap_streams = int64_t(ctx->num_sms) * nbm * gpb;  // gpb group streams per block
     } else {
       d->mw = -1;
     }
@@ -390,7 +391,7 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
   // b = 5 measured 5 % slower; this one picks the measured-better b at C2
   // and C4.)
   {
-    const int64_t per_block = mw ? 1 : 4 * segs;
+    const int64_t per_block = mw ? mw_groups_per_block(W) : 4 * segs;
     const int64_t nb = cap_streams / (int64_t(ctx->num_sms) * per_block);
     int64_t best_b = nb > 0 ? nb : 1, best_t = -1;
     for (int64_t b = nb; b >= 1 && b >= nb - 1; --b) {
@@ -426,8 +427,9 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
     if (e != cudaSuccess) return cuda_fail(ctx, e, "memset(zero row)");
   }
   const int64_t warps = (a.streams + segs - 1) / segs;
-  const int grid = mw ? int(a.streams) : int((warps + 3) / 4);
-  const int block = mw ? 32 * W : 128;
+  const int gpb = mw ? mw_groups_per_block(W) : 1;
+  const int grid = mw ? int((a.streams + gpb - 1) / gpb) : int((warps + 3) / 4);
+  const int block = mw ? 32 * W * gpb : 128;
   KRun kr;
   memset(&kr, 0, sizeof(kr));
   const int Wd = plan.width;

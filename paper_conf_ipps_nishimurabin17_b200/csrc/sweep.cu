@@ -754,24 +754,30 @@ constexpr int kMwLag = 64, kMwRing = 128, kMwSP = 16;  // boundary words per col
 // 4 warps per SMSP (128 registers) while R*S <= 44 planes of row state fit
 // without large spills; above that the register count decides.
 template <int S, int R, int W>
-constexpr int mw_min_blocks() { return R * S <= 44 ? 16 / W : 1; }
+constexpr int mw_min_blocks() { return R * S <= 44 ? 16 / (W * mw_groups_per_block(W)) : 1; }
 
 template <int S, int R, int W, int CIRC, class K>
-__global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_mw_kernel(const SweepArgs a, const K k) {
+__global__ void __launch_bounds__(32 * W * mw_groups_per_block(W), (mw_min_blocks<S, R, W>()))
+    sw_sweep_mw_kernel(const SweepArgs a, const K k) {
   constexpr int LR = 32 * R;
+  constexpr int GPB = mw_groups_per_block(W);  // group streams per block
+  static_assert(GPB <= 2, "named barriers 1 and 2 only");
   static_assert(S <= kMwSP, "boundary row holds up to 16 planes");
   const int lane = threadIdx.x & 31;
-  const int wk = threadIdx.x >> 5;  // row block of this warp
-  const int64_t stream = blockIdx.x;
-  if (stream >= a.streams) return;  // uniform per block
-  const int64_t Gs = a.base + (stream < a.rem ? 1 : 0);
-  const int64_t gb = stream * a.base + (stream < a.rem ? stream : a.rem);
+  const int gib = (threadIdx.x >> 5) / W;  // group stream of this warp within the block
+  const int wk = (threadIdx.x >> 5) % W;   // row block of this warp
+  const int64_t stream = int64_t(blockIdx.x) * GPB + gib;
 
-  __shared__ __align__(16) uint32_t bring[W - 1][kMwRing][kMwSP];
+  __shared__ __align__(16) uint32_t bring_all[GPB][W - 1][kMwRing][kMwSP];
   __shared__ __align__(16) uint32_t bzero[kMwSP];
-  __shared__ uint2 xring[W][2][32][R];
+  __shared__ uint2 xring_all[GPB][W][2][32][R];
   if (threadIdx.x < kMwSP) bzero[threadIdx.x] = 0;
   __syncthreads();
+  if (stream >= a.streams) return;  // uniform per group (its barrier is its own)
+  auto (&bring)[W - 1][kMwRing][kMwSP] = bring_all[gib];
+  auto (&xring)[W][2][32][R] = xring_all[gib];
+  const int64_t Gs = a.base + (stream < a.rem ? 1 : 0);
+  const int64_t gb = stream * a.base + (stream < a.rem ? stream : a.rem);
 
   const uint32_t nz = opaque(lane != 0 ? 1u : 0u);
   const uint32_t z0 = opaque(uint32_t(a.m) >> 31);  // 0: state reset on the FMA pipe
@@ -923,7 +929,13 @@ __global__ void __launch_bounds__(32 * W, (mw_min_blocks<S, R, W>())) sw_sweep_m
       }
       cnt -= 32;
     }
-    __syncthreads();  // phase boundary: ring writes of this phase -> reads of the next
+    // phase boundary: ring writes of this phase -> reads of the next (a named
+    // barrier per group stream, so the groups of a block do not wait on each other)
+    if (GPB == 1 || gib == 0) {  // literal barrier ids: ptxas reserves only these
+      asm volatile("bar.sync 1, %0;" ::"n"(32 * W) : "memory");
+    } else {
+      asm volatile("bar.sync 2, %0;" ::"n"(32 * W) : "memory");
+    }
   }
 }
 

@@ -1,7 +1,7 @@
 #!/usr/bin/env python3
 """Small runs of every kernel family, for compute-sanitizer.
 
-    compute-sanitizer --tool memcheck|racecheck|synccheck python tools/sanitize_run.py
+    compute-sanitizer --tool memcheck|racecheck|synccheck python tests/sanitize_run.py
 
 Each case is small (sanitizers slow kernels ~100x) but spans several groups,
 ragged pair counts and ragged lengths: the single-warp sweep (L = 16 and 32,
@@ -14,7 +14,7 @@ oracle; exits non-zero on a mismatch.
 import os
 import sys
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))  # repo root
 sys.path.insert(0, ROOT)
 
 import numpy as np  # noqa: E402

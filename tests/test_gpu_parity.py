@@ -276,8 +276,8 @@ def test_multi_device_driver():
 # ---------------------------------------------------------------- long queries (striped kernel)
 
 
-@pytest.mark.parametrize("m,n", [(257, 257), (300, 300), (384, 520), (512, 512), (700, 1000),
-                                 (1000, 700), (129, 3000), (640, 640)])
+@pytest.mark.parametrize("m,n", [(257, 257), (300, 300), (384, 520), (385, 400), (512, 512),
+                                 (700, 1000), (1000, 700), (129, 3000), (640, 640)])
 def test_long_query_lengths(m, n):
     """min(m, n) > 256: 128-row stripes handed over through the boundary buffer."""
     q, t = synth.gen_pairs(9000 + m * 7 + n, 100, m, n, planted=True)
