@@ -114,7 +114,6 @@ Layout layout(int64_t P, int mq, int nt) {
   L.G = (P + 31) / 32;
   // room for the striped / multi-warp kernels' partials: 32 lanes per 128 rows
   L.stripes = (mq + kStripeRows - 1) / kStripeRows;
-  if (L.stripes == 3) L.stripes = 4;  // multi-warp W = 3 runs as W = 4
   // the global boundary buffer is only used by the sequential striped kernel
   const bool may_stripe = mq > 512 || (mq > 128 && getenv("BPBC_NO_MULTIWARP"));
   const int64_t xbytes = (L.G * mq + kXBackPad) * 8;
@@ -218,7 +217,7 @@ struct Dispatch {
 // 512 rows (R = 4, one warp per 128 rows) and the wide-plane 129..256 case.
 int pick_mw(int mq, const Plan& p) {
   if (p.rl >= 0 || mq > 512) return -1;  // single-warp plan, or sequential stripes
-  const int W = (mq + 127) / 128 <= 2 ? 2 : 4;  // W = 3 runs as 4 (bpbc_internal.cuh)
+  const int W = (mq + 127) / 128 < 2 ? 2 : (mq + 127) / 128;  // one warp per 128 rows
   for (int i = 0; i < kNumMw; ++i)
     if (kMwR[i] == 4 && kMwW[i] == W) return i;
   return -1;
@@ -297,8 +296,11 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int nt, int c1, int c2, int g, int S
       d->L = 32;
       int nbm = 0;
       const int gpb = mw_groups_per_block(d->W);
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nbm, e.func, 32 * d->W * gpb, 0) !=
-          cudaSuccess)
+      const int smem = mw_smem_bytes(d->R, d->W);
+      if (cudaFuncSetAttribute(e.func, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) !=
+              cudaSuccess ||
+          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nbm, e.func, 32 * d->W * gpb, smem) !=
+              cudaSuccess)
         return cuda_fail(ctx, cudaGetLastError(), "occupancy");
       if (nbm < 1) nbm = 1;
       d->cap_streams = int64_t(ctx->num_sms) * nbm * gpb;  // gpb group streams per block

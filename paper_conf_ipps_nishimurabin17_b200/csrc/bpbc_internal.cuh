@@ -59,16 +59,21 @@ constexpr int kStripeRows = 32 * kStripeR;
 // Multi-warp groups (sw_sweep_mw_kernel): (R rows per lane, W warps per group)
 // (R = 2 variants splitting 128-row groups over two warps were measured
 // slower than one R = 4 warp and removed.)
-// (W = 3 runs as W = 4: a 3-warp group needs 4 groups per block to cover the
-// four schedulers, and their boundary rings exceed the 48 KB of static
-// shared memory per block.)
-constexpr int kNumMw = 2;
-constexpr int kMwR[kNumMw] = {4, 4};
-constexpr int kMwW[kNumMw] = {2, 4};
+constexpr int kNumMw = 3;
+constexpr int kMwR[kNumMw] = {4, 4, 4};
+constexpr int kMwW[kNumMw] = {2, 4, 3};
 // Groups per block of the multi-warp kernel: blocks hold a multiple of 4
 // warps so the block's warps cover the SM's four schedulers evenly (warp w of
 // a block issues from SMSP w % 4: 2- or 3-warp blocks left SMSPs idle).
 __host__ __device__ constexpr int mw_groups_per_block(int W) { return W % 4 == 0 ? 1 : W % 2 == 0 ? 2 : 4; }
+// Dynamic shared memory of a multi-warp block: per group, W - 1 boundary
+// rings of 128 columns x 16 words and the 2-slot query-plane ring (W = 3:
+// four groups, 88 KB, above the 48 KB static limit).
+constexpr int kMwRingCols = 128, kMwRingWords = 16;
+__host__ __device__ constexpr int mw_smem_bytes(int R, int W) {
+  return mw_groups_per_block(W) *
+         ((W - 1) * kMwRingCols * kMwRingWords * 4 + W * 2 * 32 * R * 8);
+}
 constexpr int kMaxShortRows = 256;     // m <= 256: the short kernel
 constexpr int64_t kMaxStripeStreams = 4096;
 constexpr int64_t kMaxBoundaryBytes = int64_t(1) << 30;

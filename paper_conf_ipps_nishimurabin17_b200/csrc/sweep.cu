@@ -749,7 +749,7 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
 // kMwRing - 33 = 95 steps after the read.  Used when a group's rows exceed one
 // warp (m > 256, or wide planes) and to put more warps on few long groups (the
 // paper's shape).  Same circuits and wavefront as the single-warp kernel.
-constexpr int kMwLag = 64, kMwRing = 128, kMwSP = 16;  // boundary words per column (padded)
+constexpr int kMwLag = 64, kMwRing = kMwRingCols, kMwSP = kMwRingWords;  // boundary words per column (padded)
 
 // 4 warps per SMSP (128 registers) while R*S <= 44 planes of row state fit
 // without large spills; above that the register count decides.
@@ -761,21 +761,25 @@ __global__ void __launch_bounds__(32 * W * mw_groups_per_block(W), (mw_min_block
     sw_sweep_mw_kernel(const SweepArgs a, const K k) {
   constexpr int LR = 32 * R;
   constexpr int GPB = mw_groups_per_block(W);  // group streams per block
-  static_assert(GPB <= 2, "named barriers 1 and 2 only");
+  static_assert(GPB <= 4, "named barriers 1..4");
   static_assert(S <= kMwSP, "boundary row holds up to 16 planes");
   const int lane = threadIdx.x & 31;
   const int gib = (threadIdx.x >> 5) / W;  // group stream of this warp within the block
   const int wk = (threadIdx.x >> 5) % W;   // row block of this warp
   const int64_t stream = int64_t(blockIdx.x) * GPB + gib;
 
-  __shared__ __align__(16) uint32_t bring_all[GPB][W - 1][kMwRing][kMwSP];
+  // dynamic shared memory (mw_smem_bytes): [GPB][W-1][ring][SP] boundary rings,
+  // then [GPB][W][2][32][R] query-plane rings
+  extern __shared__ __align__(16) uint8_t mw_smem[];
   __shared__ __align__(16) uint32_t bzero[kMwSP];
-  __shared__ uint2 xring_all[GPB][W][2][32][R];
+  using Ring = uint32_t[W - 1][kMwRing][kMwSP];
+  using XRing = uint2[W][2][32][R];
+  Ring& bring = reinterpret_cast<Ring*>(mw_smem)[gib];
+  XRing& xring = reinterpret_cast<XRing*>(mw_smem + GPB * sizeof(Ring))[gib];
+  static_assert(GPB * (sizeof(Ring) + sizeof(XRing)) == mw_smem_bytes(R, W), "smem layout");
   if (threadIdx.x < kMwSP) bzero[threadIdx.x] = 0;
   __syncthreads();
   if (stream >= a.streams) return;  // uniform per group (its barrier is its own)
-  auto (&bring)[W - 1][kMwRing][kMwSP] = bring_all[gib];
-  auto (&xring)[W][2][32][R] = xring_all[gib];
   const int64_t Gs = a.base + (stream < a.rem ? 1 : 0);
   const int64_t gb = stream * a.base + (stream < a.rem ? stream : a.rem);
 
@@ -933,18 +937,24 @@ __global__ void __launch_bounds__(32 * W * mw_groups_per_block(W), (mw_min_block
     // barrier per group stream, so the groups of a block do not wait on each other)
     if (GPB == 1 || gib == 0) {  // literal barrier ids: ptxas reserves only these
       asm volatile("bar.sync 1, %0;" ::"n"(32 * W) : "memory");
-    } else {
+    } else if (GPB == 2 || gib == 1) {
       asm volatile("bar.sync 2, %0;" ::"n"(32 * W) : "memory");
+    } else if (gib == 2) {
+      asm volatile("bar.sync 3, %0;" ::"n"(32 * W) : "memory");
+    } else {
+      asm volatile("bar.sync 4, %0;" ::"n"(32 * W) : "memory");
     }
   }
 }
 
 template <int S, int R, int W, int CIRC, class K>
 void launch_mw(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
+  // (the dispatch raised the kernel's dynamic shared memory limit, api.cu)
+  constexpr int smem = mw_smem_bytes(R, W);
   if constexpr (K::kFixed) {
-    sw_sweep_mw_kernel<S, R, W, CIRC, K><<<grid, block, 0, st>>>(a, K{});
+    sw_sweep_mw_kernel<S, R, W, CIRC, K><<<grid, block, smem, st>>>(a, K{});
   } else {
-    sw_sweep_mw_kernel<S, R, W, CIRC, KRun><<<grid, block, 0, st>>>(a, kr);
+    sw_sweep_mw_kernel<S, R, W, CIRC, KRun><<<grid, block, smem, st>>>(a, kr);
   }
 }
 
@@ -1042,6 +1052,7 @@ void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],
   reg_planes<BPBC_S, 1, true>(ptab);
   reg_mw<BPBC_S, 0>(mtab);
   reg_mw<BPBC_S, 1>(mtab);
+  reg_mw<BPBC_S, 2>(mtab);
   reg_rl<BPBC_S, 0, false>(tab);
   reg_rl<BPBC_S, 1, false>(tab);
   reg_rl<BPBC_S, 2, false>(tab);

@@ -41,7 +41,7 @@ def main():
         (40, 200, 230, (2, -1, -1), None),    # R = 8
         (50, 37, 61, (3, -2, -1), 12),        # runtime constants
         (50, 48, 80, (2, -1, -1), 5),         # saturating, fixed constants
-        (33, 300, 320, (2, -1, -1), None),    # multi-warp W = 3 -> 4
+        (33, 300, 320, (2, -1, -1), None),    # multi-warp W = 3 (4 groups per block)
         (20, 200, 240, (31, -1, -1), 13),     # multi-warp wide planes
         (9, 600, 640, (2, -1, -1), None),     # sequential stripes
     ]

@@ -284,6 +284,8 @@ def test_long_query_lengths(m, n):
     check_full(q, t)
     if min(m, n) > 256:
         assert bpbc.last_plan(0)["rows_per_lane"] == 4
+    if 256 < min(m, n) <= 512:  # multi-warp: one warp per 128 rows (W = 2..4)
+        assert bpbc.last_plan(0)["lanes"] == 32 * ((min(m, n) + 127) // 128)
 
 
 @pytest.mark.parametrize("s", [6, 8, 10, 11, 12, 16])
