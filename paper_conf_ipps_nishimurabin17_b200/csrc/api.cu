@@ -399,7 +399,9 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
     for (int64_t b = nb; b >= 1 && b >= nb - 1; --b) {
       const int64_t st_b = int64_t(ctx->num_sms) * b * per_block;
       const int64_t t = b * per_block * ((lay.G + st_b - 1) / st_b);
-      if (best_t < 0 || t < best_t) {
+      // fewer blocks only when they save more than 1 % of the work: more
+      // resident warps hide more of the circuit's dependency latency
+      if (best_t < 0 || t * 100 < best_t * 99) {
         best_t = t;
         best_b = b;
       }

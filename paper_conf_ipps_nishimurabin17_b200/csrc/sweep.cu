@@ -751,10 +751,17 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
 // paper's shape).  Same circuits and wavefront as the single-warp kernel.
 constexpr int kMwLag = 64, kMwRing = kMwRingCols, kMwSP = kMwRingWords;  // boundary words per column (padded)
 
-// 4 warps per SMSP (128 registers) while R*S <= 44 planes of row state fit
-// without large spills; above that the register count decides.
+// Resident warps per SM the register budget is sized for: 16 (128 registers)
+// while R*S <= 36 planes of row state; 12 (168 registers) up to 44, where 128
+// registers cost more in schedule than a fourth warp per SMSP gains (C5 point,
+// m = 512 at 11 bits: 4 751 vs 4 620 GCUPS; 9 bits: 16 warps 0.3 % faster);
+// above that the register count decides.
 template <int S, int R, int W>
-constexpr int mw_min_blocks() { return R * S <= 44 ? 16 / (W * mw_groups_per_block(W)) : 1; }
+constexpr int mw_min_blocks() {
+  return R * S <= 36   ? 16 / (W * mw_groups_per_block(W))
+         : R * S <= 44 ? 12 / (W * mw_groups_per_block(W))
+                       : 1;
+}
 
 template <int S, int R, int W, int CIRC, class K>
 __global__ void __launch_bounds__(32 * W * mw_groups_per_block(W), (mw_min_blocks<S, R, W>()))
