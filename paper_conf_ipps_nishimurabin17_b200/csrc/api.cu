@@ -165,14 +165,24 @@ int make_plan(int mq, int c1, int c2, int g, int S, Plan* p) {
   if (s_sat < BPBC_MIN_SCORE_BITS) s_sat = BPBC_MIN_SCORE_BITS;
   if (s_sat > S) s_sat = S;
   const int cost_sat = 11 * s_sat + 2;
-  if (spec && g >= c2) {
+  if (g >= c2) {
+    // exact offset circuit at the width no value can exceed: compile-time
+    // (+2,-1,-1) 10S LOP3, runtime constants 12S + 1 (single-warp plans
+    // only); taken when cheaper than the saturating circuit
     int s_ex = bit_length(int64_t(c1) * mq + g);
     if (s_ex < BPBC_MIN_SCORE_BITS) s_ex = BPBC_MIN_SCORE_BITS;
-    if (s_ex <= BPBC_MAX_SCORE_BITS && 10 * s_ex <= cost_sat) {
+    const int cost_ex = spec ? 10 * s_ex : 12 * s_ex + 1;
+    const int cost_sat_k = spec ? cost_sat : 13 * s_sat + 4;
+    static const bool no_exact_run = [] {  // A/B knob: BPBC_NO_EXACT_RUN=1
+      const char* v = getenv("BPBC_NO_EXACT_RUN");
+      return v != nullptr && *v != '\0' && *v != '0';
+    }();
+    const bool runtime_ok = p->rl >= 0 && !(wide_r8 && s_ex >= 13) && !no_exact_run;
+    if (s_ex <= BPBC_MAX_SCORE_BITS && cost_ex <= cost_sat_k && (spec || runtime_ok)) {
       p->circuit = kExact;
-      p->consts = kC211;
+      p->consts = spec ? kC211 : kCRun;
       p->width = s_ex;
-      p->ops = 10 * s_ex;
+      p->ops = cost_ex;
       if (wide_r8 && s_ex >= 13) {
         p->rl = -1;
         p->pad = true;
@@ -443,6 +453,10 @@ int run_device(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target, in
     kr.gmask[i] = (g >> i) & 1 ? 0xFFFFFFFFu : 0u;
   }
   kr.zmask = c2 == 0 ? 0xFFFFFFFFu : 0u;
+  for (int i = 0; i < 16; ++i) {  // exact circuit operands (used when g >= c2)
+    kr.amask[i] = ((c1 + g) >> i) & 1 ? 0xFFFFFFFFu : 0u;
+    kr.bmask[i] = g >= c2 && ((g - c2) >> i) & 1 ? 0xFFFFFFFFu : 0u;
+  }
   // threshold mode compares the diagonal term with tau (+ g for the exact
   // circuit, whose D' carries the offset g)
   const int tcmp = o.threshold + (plan.circuit == kExact ? g : 0);

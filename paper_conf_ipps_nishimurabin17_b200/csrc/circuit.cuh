@@ -109,6 +109,8 @@ struct KRun {
   uint32_t nmask[16];   // bits of (2^S - c2) mod 2^S
   uint32_t gmask[16];   // bits of g
   uint32_t zmask;       // all ones iff c2 == 0
+  uint32_t amask[16];   // exact circuit: bits of c1 + g (match operand)
+  uint32_t bmask[16];   // exact circuit: bits of g - c2 (mismatch operand, g >= c2)
 };
 
 // ---------------------------------------------------------------------------
@@ -222,9 +224,12 @@ BPBC_HD void ssub_run(const uint32_t (&X)[S], const uint32_t* gm, uint32_t (&U)[
 //   D' = diag + (e ? g - c2 : c1 + g)           one ripple adder
 //   X  = max(up, max(left, D'))                 two max_B
 //   H  = max(X - g, 0)  = max(0, up-g, left-g, diag+w)
-// kill forces H = 0 (rows past m).  LOP3 per word-cell:
-//   2 + (2S - 1) + 4S + (2S - 1) = 8S, 10S with the running max
-//   (S = 9: 90; the paper's Theorem 6 + Lemma 2 count 57S - 19 = 494).
+// kill forces H = 0 (rows past m).  LOP3 per word-cell with compile-time
+// constants: 2 + (2S - 1) + 4S + (2S - 1) = 8S, 10S with the running max
+// (S = 9: 90; the paper's Theorem 6 + Lemma 2 count 57S - 19 = 494).  With
+// runtime constants (KRun, per-bit masks): the adder operand is selected per
+// bit (+S), the gap subtract reads g's masks (3S): 10S + 1, 12S + 1 with the
+// running max (the saturating runtime circuit costs 13S + 4).
 //
 // Dp receives D' (the diagonal term).  The running maximum is taken over D'
 // instead of H (see finish_exact below), so it never waits for the
@@ -232,18 +237,28 @@ BPBC_HD void ssub_run(const uint32_t (&X)[S], const uint32_t* gm, uint32_t (&U)[
 template <int S, class K, bool KILL>
 BPBC_HD void cell_exact(const uint32_t (&up)[S], const uint32_t (&left)[S],
                         const uint32_t (&diag)[S], uint32_t xh, uint32_t xl, uint32_t yh,
-                        uint32_t yl, uint32_t kill, uint32_t (&H)[S], uint32_t (&Dp)[S]) {
-  static_assert(K::kFixed && K::g >= K::c2, "exact cell needs compile-time g >= c2");
-  constexpr int A = K::c1 + K::g, B = K::g - K::c2;
+                        uint32_t yl, uint32_t kill, uint32_t (&H)[S], uint32_t (&Dp)[S],
+                        const K& k) {
   const uint32_t e = mismatch_flag(xh, xl, yh, yl);
   uint32_t D[S];
   uint32_t c = 0u;
-  static_for<S>([&](auto I) {
-    constexpr int i = decltype(I)::value;
-    constexpr int kind = lit_kind((A >> i) & 1, (B >> i) & 1);
-    D[i] = lop3<kSumLit<kind>>(diag[i], e, c);
-    if constexpr (i + 1 < S) c = lop3<kCarryLit<kind>>(diag[i], e, c);
-  });
+  if constexpr (K::kFixed) {
+    static_assert(K::g >= K::c2, "exact cell needs g >= c2");
+    constexpr int A = K::c1 + K::g, B = K::g - K::c2;
+    static_for<S>([&](auto I) {
+      constexpr int i = decltype(I)::value;
+      constexpr int kind = lit_kind((A >> i) & 1, (B >> i) & 1);
+      D[i] = lop3<kSumLit<kind>>(diag[i], e, c);
+      if constexpr (i + 1 < S) c = lop3<kCarryLit<kind>>(diag[i], e, c);
+    });
+  } else {
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      const uint32_t w = lop3<kSel>(e, k.bmask[i], k.amask[i]);  // e ? g - c2 : c1 + g
+      D[i] = lop3<T8(TA ^ TB ^ TC)>(diag[i], w, c);
+      if (i + 1 < S) c = lop3<T8((TA & TB) | (TA & TC) | (TB & TC))>(diag[i], w, c);
+    }
+  }
   // X = max(up, max(left, D')): the inner max does not depend on `up` (the
   // previous row's fresh output), so only one comparator + mux + the gap
   // subtract sit on the row-to-row dependency chain (2S+1 deep instead of
@@ -251,7 +266,15 @@ BPBC_HD void cell_exact(const uint32_t (&up)[S], const uint32_t (&left)[S],
   uint32_t T[S], X[S];
   mux<S>(lt<S>(left, D), left, D, T);
   mux<S>(lt<S>(up, T), up, T, X);
-  ssub_const<S, K::g, KILL>(X, kill, H);
+  if constexpr (K::kFixed) {
+    ssub_const<S, K::g, KILL>(X, kill, H);
+  } else {
+    ssub_run<S>(X, k.gmask, H);
+    if constexpr (KILL) {
+#pragma unroll
+      for (int i = 0; i < S; ++i) H[i] = lop3<kAndNot>(H[i], kill, 0u);
+    }
+  }
 #pragma unroll
   for (int i = 0; i < S; ++i) Dp[i] = D[i];
 }

@@ -321,7 +321,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
       // running max over the diagonal term (circuit.cuh finish_exact); padded
       // rows are masked out of it
       if constexpr (CIRC == kExact) {
-        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn);
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn, k);
       } else {
         cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
       }
@@ -512,7 +512,7 @@ __global__ void __launch_bounds__(128) sw_sweep_planes_kernel(const SweepArgs a,
       // running max over the diagonal term (circuit.cuh finish_exact); padded
       // rows are masked out of it
       if constexpr (CIRC == kExact) {
-        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn);
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn, k);
       } else {
         cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
       }
@@ -704,7 +704,7 @@ __global__ void __launch_bounds__(128) sw_sweep_striped_kernel(const SweepArgs a
     for (int r = 0; r < R; ++r) {
       uint32_t hn[S], dn[S];
       if constexpr (CIRC == kExact) {
-        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn);
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn, k);
       } else {
         cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
       }
@@ -887,7 +887,7 @@ __global__ void __launch_bounds__(32 * W * mw_groups_per_block(W), (mw_min_block
     for (int r = 0; r < R; ++r) {
       uint32_t hn[S], dn[S];
       if constexpr (CIRC == kExact) {
-        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn);
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn, k);
       } else {
         cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
       }
@@ -1029,6 +1029,9 @@ void reg_planes(SweepEntry (*ptab)[2][13]) {
   ptab[variant_index(kSat, kCRun, PAD)][RL][S - 4] = {
       &launch_planes<S, R, L, kSat, PAD, KRun>,
       (const void*)&sw_sweep_planes_kernel<S, R, L, kSat, PAD, KRun>};
+  ptab[variant_index(kExact, kCRun, PAD)][RL][S - 4] = {
+      &launch_planes<S, R, L, kExact, PAD, KRun>,
+      (const void*)&sw_sweep_planes_kernel<S, R, L, kExact, PAD, KRun>};
 }
 
 template <int S, int RL, bool PAD>
@@ -1044,6 +1047,12 @@ void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
   tab[variant_index(kSat, kCRun, PAD)][RL][S - 4] = {
       &launch_sweep<S, R, L, kSat, PAD, KRun>,
       (const void*)&sw_sweep_kernel<S, R, L, kSat, PAD, KRun>};
+  // exact circuit with runtime constants (g >= c2; single-warp plans only)
+  if constexpr (!(RL == 3 && S >= 13)) {
+    tab[variant_index(kExact, kCRun, PAD)][RL][S - 4] = {
+        &launch_sweep<S, R, L, kExact, PAD, KRun>,
+        (const void*)&sw_sweep_kernel<S, R, L, kExact, PAD, KRun>};
+  }
 }
 
 }  // namespace

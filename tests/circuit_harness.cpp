@@ -21,6 +21,10 @@ KRun make_krun(int S, int c1, int c2, int g) {
     k.gmask[i] = (g >> i) & 1 ? 0xFFFFFFFFu : 0u;
   }
   k.zmask = c2 == 0 ? 0xFFFFFFFFu : 0u;
+  for (int i = 0; i < 16; ++i) {
+    k.amask[i] = ((c1 + g) >> i) & 1 ? 0xFFFFFFFFu : 0u;
+    k.bmask[i] = g >= c2 && ((g - c2) >> i) & 1 ? 0xFFFFFFFFu : 0u;
+  }
   return k;
 }
 
@@ -39,15 +43,19 @@ void unslice(const uint32_t (&w)[S], int* v) {
   }
 }
 
-// circuit: 0 exact (KFix<2,1,1>), 1 saturating KFix<2,1,1>, 2 saturating KRun
+// circuit: 0 exact (KFix<2,1,1>), 1 saturating KFix<2,1,1>, 2 saturating KRun,
+// 3 exact KRun (g >= c2)
 template <int S>
 void cell(int circuit, const KRun& kr, const uint32_t (&up)[S], const uint32_t (&left)[S],
           const uint32_t (&diag)[S], uint32_t xh, uint32_t xl, uint32_t yh, uint32_t yl,
           uint32_t kill, uint32_t (&H)[S], uint32_t (&D)[S]) {
   using K = KFix<2, 1, 1>;
   if (circuit == 0) {
-    if (kill) cell_exact<S, K, true>(up, left, diag, xh, xl, yh, yl, kill, H, D);
-    else cell_exact<S, K, false>(up, left, diag, xh, xl, yh, yl, 0u, H, D);
+    if (kill) cell_exact<S, K, true>(up, left, diag, xh, xl, yh, yl, kill, H, D, K{});
+    else cell_exact<S, K, false>(up, left, diag, xh, xl, yh, yl, 0u, H, D, K{});
+  } else if (circuit == 3) {
+    if (kill) cell_exact<S, KRun, true>(up, left, diag, xh, xl, yh, yl, kill, H, D, kr);
+    else cell_exact<S, KRun, false>(up, left, diag, xh, xl, yh, yl, 0u, H, D, kr);
   } else if (circuit == 1) {
     cell_sat<S, K>(up, left, diag, xh, xl, yh, yl, H, D, K{});
   } else {
@@ -86,7 +94,7 @@ long long exhaustive(int circuit, int c1, int c2, int g, int with_kill) {
       for (int d = 0; d <= cap; ++d)
         for (int e = 0; e < 2; ++e) {
           int r;
-          if (circuit == 0) {
+          if (circuit == 0 || circuit == 3) {
             // exact circuit domain: no intermediate above the cap
             if (d + c1 + g > cap || a > cap - 0 || b > cap) continue;
             r = imax(0, imax(a - g, imax(b - g, d + (e ? -c2 : c1))));
@@ -144,6 +152,10 @@ void group_dp(int circuit, int c1, int c2, int g, const uint32_t* xp, int m, con
   if (circuit == 0) {
     uint32_t F[S];
     finish_exact<S, 1>(M, F);  // KFix<2,1,1>: g = 1
+    for (int i = 0; i < S; ++i) Mout[i] = F[i];
+  } else if (circuit == 3) {  // max D' - g, floored at 0 (finish_exact with runtime g)
+    uint32_t F[S];
+    ssub_run<S>(M, kr.gmask, F);
     for (int i = 0; i < S; ++i) Mout[i] = F[i];
   } else {
     for (int i = 0; i < S; ++i) Mout[i] = M[i];

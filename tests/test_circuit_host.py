@@ -70,6 +70,18 @@ def test_sat_cell_runtime_exhaustive(harness, S, consts):
     assert harness.harness_exhaustive(2, S, c1, c2, g, 0) == 0
 
 
+@pytest.mark.parametrize("consts", [(2, 1, 1), (1, 1, 1), (3, 2, 2), (1, 3, 5), (1, 0, 0),
+                                    (2, 0, 3), (4, 1, 2)])
+@pytest.mark.parametrize("S", [4, 5, 6])
+@pytest.mark.parametrize("kill", [0, 1])
+def test_exact_cell_runtime_exhaustive(harness, S, consts, kill):
+    """Exact circuit with runtime constants (per-bit masks), any g >= c2."""
+    c1, c2, g = consts
+    if c1 + g > 2 ** S - 1:
+        pytest.skip("c1 + g must fit in S bits")
+    assert harness.harness_exhaustive(3, S, c1, c2, g, kill) == 0
+
+
 def _group_scores(harness, circuit, S, consts, q, t):
     """Run the harness DP on each 32-pair group of q/t, return untransposed scores."""
     P, m = q.shape
@@ -115,3 +127,16 @@ def test_group_dp_saturating_law(harness, S, consts):
     for circuit in ([1, 2] if consts == (2, 1, 1) else [2]):
         got = _group_scores(harness, circuit, S, consts, q, t)
         np.testing.assert_array_equal(got, want)
+
+
+@pytest.mark.parametrize("consts", [(2, 1, 1), (1, 1, 1), (3, 2, 2), (1, 3, 5), (5, 3, 4)])
+@pytest.mark.parametrize("m,n", [(5, 7), (24, 40), (40, 24)])
+def test_group_dp_exact_runtime_matches_oracle(harness, consts, m, n):
+    """Exact circuit with runtime constants at its width bit_length(c1 min(m, n) + g):
+    the group DP's max (over D', minus g) equals the oracle's score."""
+    c1, c2, g = consts
+    q, t = synth.gen_pairs(3003 + m * 7 + n + c1, 96, m, n, planted=True)
+    S = max(4, (c1 * min(m, n) + g).bit_length())
+    got = _group_scores(harness, 3, S, consts, q, t)
+    want = oracle.sw_batch(q, t, c1, -c2, -g, score_bits=S)
+    np.testing.assert_array_equal(got, want)

@@ -146,6 +146,21 @@ def test_c5_width_sweep_saturation(m, s):
     np.testing.assert_array_equal(got, np.minimum(exact, 2 ** s - 1))
 
 
+@pytest.mark.parametrize("consts", [(1, -1, -1), (3, -2, -2), (1, -3, -5), (5, -4, -4), (1, 0, 0)])
+@pytest.mark.parametrize("m,n", [(20, 40), (64, 200), (128, 128), (200, 230), (33, 1000)])
+def test_exact_circuit_runtime_constants(consts, m, n):
+    """Constants other than (+2, -1, -1) with gap >= mismatch penalty run the
+    exact offset circuit with per-bit constant masks (12S + 1 LOP3) on every
+    single-warp kernel (planes, L = 16, L = 32, R = 8)."""
+    c1, mm, g = consts
+    q, t = synth.gen_pairs(7100 + m + n + c1, 150, m, n, planted=True)
+    s = max(4, (c1 * min(m, n)).bit_length())
+    check_full(q, t, c1, mm, g, s)
+    plan = bpbc.last_plan(0)
+    assert plan["circuit"] == "exact"
+    assert plan["ops_per_word_cell"] == 12 * plan["width"] + 1
+
+
 def test_empty_batch_is_noop():
     q = torch.empty((0, 10), dtype=torch.uint8, device=DEV)
     t = torch.empty((0, 12), dtype=torch.uint8, device=DEV)
