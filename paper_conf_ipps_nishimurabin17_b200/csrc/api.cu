@@ -55,8 +55,8 @@ namespace bpbc {
 namespace {
 
 SweepEntry g_table[2][kNumVariants][kNumRL][13];  // [mode][variant][rl][S - 4]
-SweepEntry g_striped[2][3][13];                   // [mode][kind][S - 4]
-SweepEntry g_mw[2][kNumMw][3][13];                // [mode][(R, W)][kind][S - 4]
+SweepEntry g_striped[2][kNumKinds][13];           // [mode][kind][S - 4]
+SweepEntry g_mw[2][kNumMw][kNumKinds][13];        // [mode][(R, W)][kind][S - 4]
 SweepEntry g_planes[2][kNumVariants][2][13];      // [mode][variant][rl 0..1][S - 4]
 std::once_flag g_table_once;
 
@@ -167,8 +167,8 @@ int make_plan(int mq, int c1, int c2, int g, int S, Plan* p) {
   const int cost_sat = 11 * s_sat + 2;
   if (g >= c2) {
     // exact offset circuit at the width no value can exceed: compile-time
-    // (+2,-1,-1) 10S LOP3, runtime constants 12S + 1 (single-warp plans
-    // only); taken when cheaper than the saturating circuit
+    // (+2,-1,-1) 10S LOP3, runtime constants 12S + 1; taken when cheaper
+    // than the saturating circuit
     int s_ex = bit_length(int64_t(c1) * mq + g);
     if (s_ex < BPBC_MIN_SCORE_BITS) s_ex = BPBC_MIN_SCORE_BITS;
     const int cost_ex = spec ? 10 * s_ex : 12 * s_ex + 1;
@@ -177,7 +177,7 @@ int make_plan(int mq, int c1, int c2, int g, int S, Plan* p) {
       const char* v = getenv("BPBC_NO_EXACT_RUN");
       return v != nullptr && *v != '\0' && *v != '0';
     }();
-    const bool runtime_ok = p->rl >= 0 && !(wide_r8 && s_ex >= 13) && !no_exact_run;
+    const bool runtime_ok = !no_exact_run;
     if (s_ex <= BPBC_MAX_SCORE_BITS && cost_ex <= cost_sat_k && (spec || runtime_ok)) {
       p->circuit = kExact;
       p->consts = spec ? kC211 : kCRun;
@@ -267,7 +267,7 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int nt, int c1, int c2, int g, int S
   const Plan& plan = d->plan;
   d->striped = plan.rl < 0;
   d->ent = d->striped
-               ? g_striped[mode][plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]
+               ? g_striped[mode][kind_index(plan.circuit, plan.consts)]
                           [plan.width - 4]
                : g_table[mode][variant_index(plan.circuit, plan.consts, plan.pad)][plan.rl]
                         [plan.width - 4];
@@ -295,7 +295,7 @@ int make_dispatch(bpbc_sw_ctx* ctx, int mq, int nt, int c1, int c2, int g, int S
   d->mw = getenv("BPBC_NO_MULTIWARP") ? -1 : pick_mw(mq, plan);
   if (d->mw >= 0) {
     const SweepEntry e =
-        g_mw[mode][d->mw][plan.circuit == kExact ? 0 : (plan.consts == kC211 ? 1 : 2)]
+        g_mw[mode][d->mw][kind_index(plan.circuit, plan.consts)]
             [plan.width - 4];
     if (e.launch) {
       d->ent = e;

@@ -19,6 +19,12 @@ constexpr int64_t kYBackPadExtra = 640;
 enum Circuit : int { kExact = 0, kSat = 1 };
 enum Mode : int { kModeMax = 0, kModeThreshold = 1 };  // running max / sticky flag
 enum Consts : int { kC211 = 0, kCRun = 1 };
+// Kernel kinds of the multi-warp and striped registries: exact (+2,-1,-1),
+// saturating (+2,-1,-1), saturating runtime constants, exact runtime constants.
+constexpr int kNumKinds = 4;
+constexpr int kind_index(int circuit, int consts) {
+  return circuit == kExact ? (consts == kC211 ? 0 : 3) : (consts == kC211 ? 1 : 2);
+}
 constexpr int kNumVariants = 8;  // circuit x consts x padded-rows
 constexpr int variant_index(int circuit, int consts, bool pad) {
   return (circuit * 2 + consts) * 2 + (pad ? 1 : 0);
@@ -97,9 +103,9 @@ SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
 // (+2,-1,-1), 2 saturating runtime constants).
 #define BPBC_DECLARE_REG(S)                                                       \
   void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
-                                SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]);    \
+                                SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13]);    \
   void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
-                                SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]);
+                                SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13]);
 BPBC_DECLARE_REG(4)
 BPBC_DECLARE_REG(5)
 BPBC_DECLARE_REG(6)

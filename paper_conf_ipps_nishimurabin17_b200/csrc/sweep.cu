@@ -966,7 +966,7 @@ void launch_mw(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStre
 }
 
 template <int S, int MV>
-void reg_mw(SweepEntry (*mtab)[3][13]) {
+void reg_mw(SweepEntry (*mtab)[kNumKinds][13]) {
   constexpr int R = kMwR[MV], W = kMwW[MV];
   using K211 = KFix<2, 1, 1>;
   mtab[MV][0][S - 4] = {&launch_mw<S, R, W, kExact, K211>,
@@ -975,6 +975,8 @@ void reg_mw(SweepEntry (*mtab)[3][13]) {
                         (const void*)&sw_sweep_mw_kernel<S, R, W, kSat, K211>};
   mtab[MV][2][S - 4] = {&launch_mw<S, R, W, kSat, KRun>,
                         (const void*)&sw_sweep_mw_kernel<S, R, W, kSat, KRun>};
+  mtab[MV][3][S - 4] = {&launch_mw<S, R, W, kExact, KRun>,
+                        (const void*)&sw_sweep_mw_kernel<S, R, W, kExact, KRun>};
 }
 
 template <int S, int R, int L, int CIRC, bool PAD, class K>
@@ -1005,6 +1007,8 @@ void reg_striped(SweepEntry (*stab)[13]) {
                     (const void*)&sw_sweep_striped_kernel<S, kSat, K211, R>};
   stab[2][S - 4] = {&launch_striped<S, kSat, KRun, R>,
                     (const void*)&sw_sweep_striped_kernel<S, kSat, KRun, R>};
+  stab[3][S - 4] = {&launch_striped<S, kExact, KRun, R>,
+                    (const void*)&sw_sweep_striped_kernel<S, kExact, KRun, R>};
 }
 
 template <int S, int R, int L, int CIRC, bool PAD, class K>
@@ -1061,7 +1065,7 @@ void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
 #define BPBC_CAT(a, b) BPBC_CAT2(a, b)
 #define BPBC_REGNAME BPBC_CAT(BPBC_CAT(BPBC_CAT(register_sweep_s, BPBC_S), _m), BPBC_MODE)
 void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],
-                  SweepEntry (*mtab)[3][13], SweepEntry (*ptab)[2][13]) {
+                  SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13]) {
   reg_planes<BPBC_S, 0, false>(ptab);
   reg_planes<BPBC_S, 1, false>(ptab);
   reg_planes<BPBC_S, 0, true>(ptab);

@@ -44,6 +44,9 @@ def main():
         (33, 300, 320, (2, -1, -1), None),    # multi-warp W = 3 (4 groups per block)
         (20, 200, 240, (31, -1, -1), 13),     # multi-warp wide planes
         (9, 600, 640, (2, -1, -1), None),     # sequential stripes
+        (40, 100, 130, (3, -2, -2), None),    # exact circuit, runtime constants
+        (33, 300, 320, (1, -1, -1), None),    # ... multi-warp W = 3
+        (9, 600, 640, (1, -3, -5), None),     # ... sequential stripes
     ]
     for P, m, n, (c1, mm, g), s in cases:
         q, t = synth.gen_pairs(4000 + m + n, P, m, n, planted=True)

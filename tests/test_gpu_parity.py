@@ -147,11 +147,13 @@ def test_c5_width_sweep_saturation(m, s):
 
 
 @pytest.mark.parametrize("consts", [(1, -1, -1), (3, -2, -2), (1, -3, -5), (5, -4, -4), (1, 0, 0)])
-@pytest.mark.parametrize("m,n", [(20, 40), (64, 200), (128, 128), (200, 230), (33, 1000)])
+@pytest.mark.parametrize("m,n", [(20, 40), (64, 200), (128, 128), (200, 230), (33, 1000),
+                                 (300, 310), (512, 520), (600, 640)])
 def test_exact_circuit_runtime_constants(consts, m, n):
     """Constants other than (+2, -1, -1) with gap >= mismatch penalty run the
     exact offset circuit with per-bit constant masks (12S + 1 LOP3) on every
-    single-warp kernel (planes, L = 16, L = 32, R = 8)."""
+    kernel family (planes, L = 16, L = 32, R = 8, multi-warp W = 3 / 4,
+    sequential stripes)."""
     c1, mm, g = consts
     q, t = synth.gen_pairs(7100 + m + n + c1, 150, m, n, planted=True)
     s = max(4, (c1 * min(m, n)).bit_length())
