@@ -35,7 +35,18 @@
  *   - asynchronous functions only ENQUEUE work on `stream` (a cudaStream_t,
  *     NULL = legacy default stream) and return; the caller keeps every
  *     buffer alive until the stream has completed that work;
- *   - a ctx is not thread-safe: use one ctx per device per host thread.
+ *   - no function synchronizes the whole device: the blocking ones wait
+ *     only for work this ctx enqueued;
+ *   - ctx-owned buffers (the workspace used when `workspace` is NULL) are
+ *     ordered across streams by the library: a call on stream B after a
+ *     call on stream A makes B wait for A's use of them (an event), so
+ *     calls on different streams through one ctx never share them
+ *     concurrently.  Caller-owned workspaces are the caller's to order
+ *     (give concurrent streams separate workspaces);
+ *   - a ctx is not thread-safe: use one ctx per device per host thread;
+ *   - the environment is read once, in bpbc_sw_init (benchmark knobs only:
+ *     BPBC_MAX_BLOCKS_PER_SM, BPBC_NO_EXACT_RUN, BPBC_WRAP); no call on the
+ *     hot path reads it.
  */
 #ifndef BPBC_SW_H
 #define BPBC_SW_H
@@ -55,7 +66,8 @@ typedef enum {
     BPBC_ERR_UNSUPPORTED = -2, /* valid but outside what this build supports     */
     BPBC_ERR_CUDA = -3,        /* a CUDA call failed; text in bpbc_sw_last_error */
     BPBC_ERR_OOM = -4,         /* device or host allocation failed               */
-    BPBC_ERR_BAD_BASE = -5     /* reported by bpbc_sw_check_flags               */
+    BPBC_ERR_BAD_BASE = -5     /* returned by bpbc_sw_get_error_flags when a base
+                                  code > 3 was seen since the last read */
 } bpbc_status;
 
 /* Sticky device flags (bpbc_sw_get_error_flags). */
@@ -67,22 +79,36 @@ typedef enum {
 #define BPBC_MAX_LEN (1 << 20)       /* m, n <= 2^20 */
 #define BPBC_MAX_QUERY_LEN (1 << 16) /* min(m, n) <= 2^16 */
 
-/* Binds the context to `cuda_device`, creates its device flag word and
- * queries the SM count.  No pair-sized allocation.  *out_ctx is set only on
- * success. */
+/* Binds the context to `cuda_device`, creates its device flag word, a
+ * private stream for flag reads and queries the SM count; reads the
+ * benchmark knobs from the environment (once).  No pair-sized allocation.
+ * *out_ctx is set only on success. */
 int bpbc_sw_init(int cuda_device, bpbc_sw_ctx **out_ctx);
 
-/* Frees everything the ctx owns (its lazily grown workspace and host
- * staging buffers).  Synchronizes the device first.  NULL is a no-op. */
+/* Waits for the work this ctx enqueued (on every stream it used), then frees
+ * everything the ctx owns (workspace, host-path buffers and streams, pinned
+ * staging).  NULL is a no-op. */
 int bpbc_sw_destroy(bpbc_sw_ctx *ctx);
 
-/* Bytes of device workspace bpbc_sw_score_batch needs for these sizes:
- * the bit-transposed planes 8 * ceil(P/32) * (m + n) bytes plus padding,
- * the per-lane partial maxima (2 KiB per 32-pair group, per 128 query rows
- * when min(m, n) > 256) and, when min(m, n) > 256, the stripe boundary rows
- * (64 * max(m, n) bytes per concurrent group stream, at most 1 GiB).  Pure
- * host function. */
+/* Upper bound on the device workspace any bpbc_sw_score_batch* /
+ * bpbc_sw_filter_batch call with these sizes needs, whatever its constants
+ * and width: the bit-transposed planes 8 * ceil(P/32) * (m + n) bytes plus
+ * padding (only plans that run the separate pack pass use them), the
+ * per-lane partial maxima (2 KiB per 32-pair group, per 128 query rows), the
+ * stripe boundary rows when min(m, n) > 128 (64 * max(m, n) bytes per
+ * concurrent group stream, at most 1 GiB), the wrap-around schedule's warp
+ * snapshots when the batch has few groups (<= 8192) of a long target, and the
+ * filter's compaction scratch.  Pure host function. */
 int bpbc_sw_workspace_bytes(int64_t num_pairs, int32_t m, int32_t n, size_t *bytes);
+
+/* Exact device workspace of one call with these arguments (the plan the
+ * call will run on ctx's device: circuit, kernel, schedule), <= the bound
+ * above.  filter != 0: for bpbc_sw_filter_batch.  Errors as
+ * bpbc_sw_score_batch's argument checks.  Host function (queries the
+ * kernels' occupancy once). */
+int bpbc_sw_workspace_bytes_for(bpbc_sw_ctx *ctx, int64_t num_pairs, int32_t m, int32_t n,
+                                int32_t match, int32_t mismatch, int32_t gap,
+                                int32_t score_bits, int32_t filter, size_t *bytes);
 
 /*
  * The hot path (Steps 2-4): pack (W2B) -> bit-sliced wavefront
@@ -103,9 +129,10 @@ int bpbc_sw_workspace_bytes(int64_t num_pairs, int32_t m, int32_t n, size_t *byt
  *             -mismatch and -gap must each be <= 2^s - 1.  Results are
  *             min(score, 2^s - 1) exactly (R3).
  * out_scores  device, int32 [num_pairs].
- * workspace   device scratch of >= bpbc_sw_workspace_bytes(...) bytes owned
- *             by the caller, or NULL to use a ctx-owned buffer grown on
- *             demand (allocation happens on the calling thread).
+ * workspace   device scratch owned by the caller of >= bpbc_sw_workspace_bytes_for
+ *             (...) bytes (bpbc_sw_workspace_bytes is always enough), or NULL
+ *             to use the ctx-owned buffer, grown on demand in stream order
+ *             (cudaMallocAsync on `stream`; no device-wide sync).
  * stream      cudaStream_t to enqueue on.
  *
  * Errors (host-side, no device sync): INVALID_ARG for negative sizes, NULL
@@ -123,9 +150,15 @@ int bpbc_sw_score_batch(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8_t *t
 /*
  * End-to-end variant with HOST buffers (the paper's Steps 1-5):
  * copies the inputs host->device, runs the hot path and copies the scores
- * device->host, chunked over pair ranges so copies of one chunk overlap the
- * kernels of the previous one.  Blocking: returns when out_scores is
- * written.  Uses ctx-owned device buffers.
+ * device->host.  The batch is cut into chunks of whole waves (one 32-pair
+ * group per resident sweep stream) that flow through three ctx-owned
+ * buffer slots on three ctx-owned streams (copy-in, kernels, copy-out), so
+ * the copy of chunk c+1 and the result copy of chunk c-1 overlap the kernels
+ * of chunk c.  The chunk plan uses the H2D and cell rates this ctx measured
+ * on its previous host call.  Batches with few groups (the wrap-around
+ * schedule) run as one chunk.  Pinned inputs overlap (pageable ones are
+ * staged by the driver); a pageable out_scores goes through pinned staging.
+ * Blocking: returns when out_scores is written.
  *
  * query, target  host, uint8 [num_pairs][m] / [num_pairs][n].
  * out_scores     host, int32 [num_pairs].
@@ -171,7 +204,8 @@ int bpbc_sw_score_batch_host_packed2(bpbc_sw_ctx *ctx, const uint8_t *query2,
  * out_indices  device, int64 [num_pairs] or NULL: the flagged pair indices in
  *              ascending order (the first *out_count entries are written).
  * out_count    device, int64 [1] or NULL: number of flagged pairs.
- * The compaction uses ctx-owned scratch (grown on demand).  Other arguments
+ * The compaction scratch is a section of the workspace (size it with
+ * bpbc_sw_workspace_bytes_for(..., filter = 1, ...)).  Other arguments
  * and errors as bpbc_sw_score_batch; a threshold outside the range above is
  * INVALID_ARG.  Asynchronous on `stream`.
  */
@@ -220,8 +254,11 @@ int bpbc_sw_untranspose(bpbc_sw_ctx *ctx, const uint32_t *partial, int64_t num_g
                         int32_t lanes, int32_t s, int64_t num_pairs, int32_t cap,
                         int32_t *out, void *stream);
 
-/* Synchronizes the ctx's device, returns the sticky flags in *flags (bit 0 =
- * BPBC_FLAG_BAD_BASE) and clears them. */
+/* Waits for the work this ctx enqueued on every stream it used since the
+ * last read (not the whole device), returns the sticky flags in *flags (bit
+ * 0 = BPBC_FLAG_BAD_BASE) and clears them.  Returns BPBC_ERR_BAD_BASE when
+ * that bit was set (the scores of those calls used c & 3 for the bad codes,
+ * R18), BPBC_OK otherwise; *flags is written in both cases. */
 int bpbc_sw_get_error_flags(bpbc_sw_ctx *ctx, uint32_t *flags);
 
 /* Description of the last sweep dispatch (for benchmarks and tests):
@@ -238,6 +275,13 @@ int bpbc_sw_last_plan(bpbc_sw_ctx *ctx, int32_t *circuit, int32_t *width, int32_
  * kernel that transposes the raw codes itself (1) or ran on packed planes
  * (0).  Either pointer may be NULL. */
 int bpbc_sw_last_launches(bpbc_sw_ctx *ctx, int32_t *kernels, int32_t *fused);
+
+/* Stream schedule of the last sweep: wrap = 1 if it used the wrap-around
+ * schedule (streams take equal runs of the concatenated target columns and
+ * hand split groups over as warp-state snapshots), 0 for the
+ * group-granular split; blocks_per_sm = resident sweep blocks per SM the
+ * plan chose.  Either pointer may be NULL. */
+int bpbc_sw_last_schedule(bpbc_sw_ctx *ctx, int32_t *wrap, int64_t *blocks_per_sm);
 
 /* Per-phase device timing, the columns of the paper's Table IV (P:L384-413:
  * W2B, SWA, B2W).  bpbc_sw_profile(ctx, 1) clears the accumulators and makes

@@ -31,6 +31,9 @@ SIGNATURES = {
     "bpbc_sw_destroy": (_c.c_int, [_vp]),
     "bpbc_sw_workspace_bytes": (_c.c_int, [_c.c_int64, _c.c_int32, _c.c_int32,
                                            _c.POINTER(_c.c_size_t)]),
+    "bpbc_sw_workspace_bytes_for": (_c.c_int, [_vp, _c.c_int64, _c.c_int32, _c.c_int32,
+                                               _c.c_int32, _c.c_int32, _c.c_int32, _c.c_int32,
+                                               _c.c_int32, _c.POINTER(_c.c_size_t)]),
     "bpbc_sw_score_batch": (_c.c_int, [_vp, _vp, _vp, _c.c_int64, _c.c_int32, _c.c_int32,
                                        _c.c_int32, _c.c_int32, _c.c_int32, _c.c_int32, _vp,
                                        _vp, _c.c_size_t, _vp]),
@@ -58,6 +61,7 @@ SIGNATURES = {
                                      _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int32),
                                      _c.POINTER(_c.c_int64), _c.POINTER(_c.c_int32)]),
     "bpbc_sw_last_launches": (_c.c_int, [_vp, _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int32)]),
+    "bpbc_sw_last_schedule": (_c.c_int, [_vp, _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int64)]),
     "bpbc_sw_profile": (_c.c_int, [_vp, _c.c_int]),
     "bpbc_sw_profile_read": (_c.c_int, [_vp, _c.POINTER(_c.c_double), _c.POINTER(_c.c_int64)]),
     "bpbc_sw_status_string": (_c.c_char_p, [_c.c_int]),

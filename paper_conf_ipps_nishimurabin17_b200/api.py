@@ -39,6 +39,16 @@ def destroy_all() -> None:
         _ctxs.clear()
 
 
+def release_thread_ctx(device: int) -> None:
+    """Destroy the calling thread's ctx for ``device`` (worker threads call
+    this before they exit, so their device buffers do not outlive them)."""
+    key = (device, threading.get_ident())
+    with _ctx_lock:
+        c = _ctxs.pop(key, None)
+    if c is not None:
+        _lib.load().bpbc_sw_destroy(c)
+
+
 def default_score_bits(match: int, m: int, n: int) -> int:
     """s = bit_length(match * min(m, n)) (reading R2), in [4, 16]."""
     return min(16, max(4, (match * min(m, n)).bit_length()))
@@ -51,8 +61,23 @@ def _stream_ptr(stream, device) -> int:
 
 
 def workspace_bytes(num_pairs: int, m: int, n: int) -> int:
+    """bpbc_sw_workspace_bytes: upper bound over every plan of these sizes."""
     v = ctypes.c_size_t()
     check(_lib.load().bpbc_sw_workspace_bytes(num_pairs, m, n, ctypes.byref(v)))
+    return v.value
+
+
+def workspace_bytes_for(num_pairs: int, m: int, n: int, match: int = 2, mismatch: int = -1,
+                        gap: int = -1, score_bits: int | None = None, filter: bool = False,
+                        device: int = 0) -> int:
+    """bpbc_sw_workspace_bytes_for: the exact workspace of that call on ``device``."""
+    if score_bits is None:
+        score_bits = default_score_bits(match, m, n)
+    v = ctypes.c_size_t()
+    ctx = _ctx(device)
+    check(_lib.load().bpbc_sw_workspace_bytes_for(ctx, num_pairs, m, n, match, mismatch, gap,
+                                                  score_bits, int(bool(filter)),
+                                                  ctypes.byref(v)), ctx)
     return v.value
 
 
@@ -131,9 +156,13 @@ def filter_batch(query: torch.Tensor, target: torch.Tensor, threshold: int, matc
     dev = query.device.index if query.device.index is not None else torch.cuda.current_device()
     if score_bits is None:
         score_bits = default_score_bits(match, m, n)
-    mask = torch.empty((P + 31) // 32, dtype=torch.int32, device=query.device)
-    count = torch.zeros(1, dtype=torch.int64, device=query.device)
-    idx = torch.empty(P, dtype=torch.int64, device=query.device) if indices else None
+    # outputs are allocated on the stream the C call writes them on (the C
+    # side writes every count / mask word, no zero fill needed)
+    st = stream if stream is not None else torch.cuda.current_stream(query.device)
+    with torch.cuda.stream(st):
+        mask = torch.empty((P + 31) // 32, dtype=torch.int32, device=query.device)
+        count = torch.empty(1, dtype=torch.int64, device=query.device)
+        idx = torch.empty(P, dtype=torch.int64, device=query.device) if indices else None
     ws_ptr, ws_bytes = None, 0
     if workspace is not None:
         ws_ptr, ws_bytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
@@ -141,7 +170,7 @@ def filter_batch(query: torch.Tensor, target: torch.Tensor, threshold: int, matc
     check(_lib.load().bpbc_sw_filter_batch(
         ctx, query.data_ptr(), target.data_ptr(), P, m, n, match, mismatch, gap, score_bits,
         threshold, mask.data_ptr(), idx.data_ptr() if idx is not None else None,
-        count.data_ptr(), ws_ptr, ws_bytes, _stream_ptr(stream, query.device)), ctx)
+        count.data_ptr(), ws_ptr, ws_bytes, st.cuda_stream), ctx)
     return mask, count, idx
 
 
@@ -249,10 +278,21 @@ def untranspose(partial: torch.Tensor, num_pairs: int, cap: int, stream=None) ->
 
 
 def get_error_flags(device: int = 0) -> int:
+    """bpbc_sw_get_error_flags: the sticky flags since the last read (bit 0 =
+    BPBC_FLAG_BAD_BASE), cleared.  The C call returns BPBC_ERR_BAD_BASE when
+    that bit is set; here the bit is returned (check_flags raises)."""
     v = ctypes.c_uint32()
     ctx = _ctx(device)
-    check(_lib.load().bpbc_sw_get_error_flags(ctx, ctypes.byref(v)), ctx)
+    rc = _lib.load().bpbc_sw_get_error_flags(ctx, ctypes.byref(v))
+    if rc not in (_lib.BPBC_OK, _lib.BPBC_ERR_BAD_BASE):
+        check(rc, ctx)
     return v.value
+
+
+def check_flags(device: int = 0) -> None:
+    """Raise BPBCError(BPBC_ERR_BAD_BASE) if a base code > 3 was seen."""
+    if get_error_flags(device) & _lib.BPBC_FLAG_BAD_BASE:
+        raise _lib.BPBCError(_lib.BPBC_ERR_BAD_BASE, "a base code > 3 was read as c & 3")
 
 
 def last_plan(device: int = 0) -> dict:
@@ -264,10 +304,12 @@ def last_plan(device: int = 0) -> dict:
                                         ctypes.byref(o)))
     k, f = ctypes.c_int32(), ctypes.c_int32()
     check(_lib.load().bpbc_sw_last_launches(_ctx(device), ctypes.byref(k), ctypes.byref(f)))
+    wr, bps = ctypes.c_int32(), ctypes.c_int64()
+    check(_lib.load().bpbc_sw_last_schedule(_ctx(device), ctypes.byref(wr), ctypes.byref(bps)))
     return {"circuit": ["exact", "saturating"][c.value] if c.value >= 0 else None,
             "width": w.value, "rows_per_lane": r.value, "lanes": l.value,
             "streams": s.value, "ops_per_word_cell": o.value, "kernels": k.value,
-            "fused": bool(f.value)}
+            "fused": bool(f.value), "wrap": bool(wr.value), "blocks_per_sm": bps.value}
 
 
 def profile(enable: bool, device: int = 0) -> None:

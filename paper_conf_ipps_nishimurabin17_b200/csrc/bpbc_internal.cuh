@@ -56,7 +56,26 @@ struct SweepArgs {
   int stripes;          // row stripes of kStripeRows per group (1 = short kernel)
   uint32_t* bnd;        // [streams][n][SP] stripe boundary rows
   const uint32_t* bzero;  // 16 zero words
+  // Wrap-around schedule (fused single-warp kernel, L = 32, n % 32 == 0;
+  // DESIGN.md 6.2): stream k owns the columns [k span, (k+1) span) of the
+  // concatenation of all groups' columns (group g, column j -> g n + j),
+  // processed as head piece -> whole groups -> tail piece; a group split
+  // between two streams moves its whole warp state (a snapshot) through
+  // `snap` once the earlier stream has finished its head.
+  int wrap;             // 1: wrap-around schedule (streams = ceil(G n / span))
+  int64_t span;         // columns per stream (multiple of 32, >= n)
+  uint32_t* snap;       // [streams][kSnapWords][32] warp-state snapshots
+  uint32_t* snap_flag;  // [streams] 1 once snapshot k is written (zeroed per call)
 };
+
+// Words of one lane's warp-state snapshot (wrap-around schedule): R rows x S
+// planes of scores, S planes of the diagonal input, S planes of running max
+// (or the threshold flag word).
+__host__ __device__ constexpr int snap_words(int R, int S) { return (R + 2) * S; }
+// The wrap-around schedule's groups bound (above it the group-granular split
+// wastes < 1 %); snapshot slots are reserved for at most kWrapMaxStreams.
+constexpr int64_t kWrapMaxGroups = 8192;
+constexpr int64_t kWrapMaxStreams = 4096;
 
 // Long queries: stripes of kStripeR rows per lane x 32 lanes (R = 2 stripes
 // were measured 1.7x slower at C5).
@@ -100,12 +119,16 @@ SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
 // Registration hooks, one per (score width, mode): sweep.cu is compiled once
 // per pair with -DBPBC_S=S -DBPBC_MODE=M.  tab: [variant][rl][S-4] of the
 // short kernel, stab: [striped kind][S-4] (0 exact (+2,-1,-1), 1 saturating
-// (+2,-1,-1), 2 saturating runtime constants).
+// (+2,-1,-1), 2 saturating runtime constants), ptab: [variant][rl 0..1][S-4]
+// of the planes kernel, wtab: [variant][rl - 2][S-4] of the wrap-around
+// kernel (L = 32 tilings).
 #define BPBC_DECLARE_REG(S)                                                       \
   void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
-                                SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13]);    \
+                                SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13], \
+                                SweepEntry (*wtab)[2][13]);                                   \
   void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
-                                SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13]);
+                                SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13], \
+                                SweepEntry (*wtab)[2][13]);
 BPBC_DECLARE_REG(4)
 BPBC_DECLARE_REG(5)
 BPBC_DECLARE_REG(6)

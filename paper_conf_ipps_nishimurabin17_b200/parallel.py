@@ -96,11 +96,12 @@ def score_sharded(query: torch.Tensor, target: torch.Tensor, num_pairs: int, mat
 def score_multi_device(query: np.ndarray, target: np.ndarray, match: int = 2,
                        mismatch: int = -1, gap: int = -1, score_bits: int | None = None,
                        devices: list[int] | None = None,
-                       out: np.ndarray | None = None) -> np.ndarray:
+                       out: np.ndarray | None = None, return_flags: bool = False):
     """Host arrays in, host int32 scores out, sharded over ``devices`` (one
-    host thread and one ctx per device, each running the blocking
-    host-buffer C call on its slice).  A failing shard raises with its
-    device id."""
+    host thread per device, each with its own ctx that is destroyed when the
+    thread ends, running the blocking host-buffer C call on its slice).  A
+    failing shard raises with its device id.  return_flags=True also returns
+    each shard's sticky error flags (bit 0 = a base code > 3)."""
     query = np.ascontiguousarray(query, dtype=np.uint8)
     target = np.ascontiguousarray(target, dtype=np.uint8)
     P, m = query.shape
@@ -114,6 +115,7 @@ def score_multi_device(query: np.ndarray, target: np.ndarray, match: int = 2,
     if out is None:
         out = np.empty(P, dtype=np.int32)
     errors: dict[int, BaseException] = {}
+    flags = [0] * len(devices)
 
     def work(rank, dev):
         b, e = shard_range(P, len(devices), rank)
@@ -122,8 +124,12 @@ def score_multi_device(query: np.ndarray, target: np.ndarray, match: int = 2,
         try:
             api.score_batch_host(query[b:e], target[b:e], match, mismatch, gap, score_bits,
                                  device=dev, out=out[b:e])
+            flags[rank] = api.get_error_flags(dev)
         except BaseException as exc:  # re-raised below with the device id
             errors[dev] = exc
+        finally:
+            # this thread's ctx (and its shard-sized device buffers) ends with it
+            api.release_thread_ctx(dev)
 
     threads = [threading.Thread(target=work, args=(r, d)) for r, d in enumerate(devices)]
     for t in threads:
@@ -133,4 +139,6 @@ def score_multi_device(query: np.ndarray, target: np.ndarray, match: int = 2,
     if errors:
         dev, exc = next(iter(errors.items()))
         raise RuntimeError(f"shard on cuda:{dev} failed: {exc}") from exc
+    if return_flags:
+        return out, flags
     return out

@@ -1,0 +1,36 @@
+#!/bin/bash
+# One parametrised recipe for the GPU box (replaces the round-1 one-off
+# tools/gpu_run*.sh scripts).  Run through gpurun from the repo root, e.g.
+#   gpurun --timeout 1200 -- 'bash tools/gpu.sh TAG tests bench ncu:"--config 5 --m 32 --n 32 --score-bits 7"'
+# Every artefact lands in gpurun_out/TAG_*.  Steps (in the order given):
+#   tests            pytest -m gpu (junit + log)
+#   smoke            __graft_entry__.smoke()
+#   bench[:ARGS]     python bench.py ARGS (default: the driver's N=1 command)
+#   launches[:ARGS]  ncu launch list (gpu__time_duration, clocks not locked) of bench.py ARGS
+#   ncu[:ARGS]       ncu --set full --import-source of the first sweep launch of bench.py ARGS
+#   sanitize         compute-sanitizer memcheck/racecheck/synccheck/initcheck over tests/sanitize_run.py
+#   py:FILE[:ARGS]   python FILE ARGS
+set -u
+tag=$1; shift
+out=gpurun_out
+mkdir -p $out
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,temperature.gpu --format=csv > $out/${tag}_gpu.txt 2>&1
+i=0
+for step in "$@"; do
+  i=$((i + 1))
+  kind=${step%%:*}
+  args=""
+  [ "$kind" != "$step" ] && args=${step#*:}
+  echo "== [$i] $kind $args" | tee -a $out/${tag}_steps.log
+  case $kind in
+    tests) timeout 2400 python -m pytest tests -m gpu -q -x --junitxml=$out/${tag}_junit.xml > $out/${tag}_tests.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
+    smoke) timeout 600 python -c 'import __graft_entry__ as g; g.smoke()' > $out/${tag}_smoke.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
+    bench) timeout 1800 python bench.py $args > $out/${tag}_bench$i.json 2> $out/${tag}_bench$i.err; echo "rc=$?" >> $out/${tag}_steps.log ;;
+    launches) timeout 1800 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $out/${tag}_launches$i.csv python bench.py $args > $out/${tag}_launches$i.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
+    ncu) timeout 1800 ncu --set full --clock-control none --import-source on -k regex:sw_sweep -c 1 -o $out/${tag}_full$i python bench.py $args > $out/${tag}_ncu$i.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
+    sanitize) for tool in memcheck racecheck synccheck initcheck; do timeout 1200 compute-sanitizer --tool $tool python tests/sanitize_run.py > $out/${tag}_san_$tool.log 2>&1; echo "$tool rc=$?" >> $out/${tag}_steps.log; done ;;
+    py) f=${args%%:*}; a=""; [ "$f" != "$args" ] && a=${args#*:}; timeout 2400 python $f $a > $out/${tag}_py$i.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
+    *) echo "unknown step $kind" >> $out/${tag}_steps.log ;;
+  esac
+done
+echo done >> $out/${tag}_steps.log
