@@ -251,12 +251,18 @@ def score_batch_host_packed2(query2: np.ndarray, target2: np.ndarray, m: int, n:
     return out
 
 
-def pack(codes: torch.Tensor, stream=None) -> torch.Tensor:
-    """bpbc_sw_pack: uint8 [P, len] -> uint32 [ceil(P/32), len, 2] bit planes (H, L)."""
+def pack(codes: torch.Tensor, stream=None, out: torch.Tensor | None = None) -> torch.Tensor:
+    """bpbc_sw_pack: uint8 [P, len] -> uint32 [ceil(P/32), len, 2] bit planes (H, L)
+    (returned as an int32 view; ``out`` may supply that tensor)."""
     codes = codes.contiguous()
     P, ln = codes.shape
     G = (P + 31) // 32
-    planes = torch.empty((G, ln, 2), dtype=torch.int32, device=codes.device)
+    if out is not None:
+        if out.shape != (G, ln, 2) or out.dtype != torch.int32 or not out.is_contiguous():
+            raise ValueError(f"out must be a contiguous int32 [{G}, {ln}, 2] tensor")
+        planes = out
+    else:
+        planes = torch.empty((G, ln, 2), dtype=torch.int32, device=codes.device)
     dev = codes.device.index or 0
     ctx = _ctx(dev)
     check(_lib.load().bpbc_sw_pack(ctx, codes.data_ptr(), P, ln, planes.data_ptr(),

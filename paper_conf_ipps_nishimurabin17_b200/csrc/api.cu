@@ -790,28 +790,36 @@ int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t*
     return rc;
   // (few groups: a chunk of them would leave SMSPs idle -- no chunking)
   const int64_t wave_pairs = full.wrap ? num_pairs : full.streams * 32;
-  // Chunk plan from the measured rates: copy-bound (H2D time per pair >=
-  // compute time per pair) -> ~12 equal chunks, so the last chunk's kernels
-  // are short; compute-bound -> chunks growing 1, 2, 4, ... waves, so the
-  // first copy is short.
+  // Chunk plan from the measured rates.  Every chunk's
+  // kernels pay one pipeline fill / drain (~L steps per stream), so chunks
+  // are few and large:
+  //  * copy-bound (H2D time per pair >= kernel time per pair): ~12 equal
+  //    chunks -- the run takes the whole copy plus the last chunk's kernels;
+  //  * compute-bound: chunks growing geometrically from one wave, by the
+  //    factor the kernels outpace the copy (the copy of chunk c+1 hides
+  //    under the kernels of chunk c), capped at 4x.
   const double h2d_s = double(qs + ts) / ctx->h2d_bps;
   const double comp_s = double(mq) * nt / ctx->cells_ps;
+  const int64_t waves = ceil_div(num_pairs, wave_pairs);
   std::vector<int64_t> bounds{0};
   if (h2d_s >= comp_s) {
-    const int64_t waves = ceil_div(num_pairs, wave_pairs);
     const int64_t per = ceil_div(waves, 12);
     while (bounds.back() < num_pairs) {
       const int64_t left = num_pairs - bounds.back();
       bounds.push_back(bounds.back() + (left < per * wave_pairs ? left : per * wave_pairs));
     }
   } else {
-    const int64_t waves = ceil_div(num_pairs, wave_pairs);
-    const int64_t cap_w = waves / 6 > 1 ? waves / 6 : 1;  // at least ~6 chunks when possible
-    for (int64_t w = 1; bounds.back() < num_pairs; w = w * 2 < cap_w ? w * 2 : cap_w) {
+    double f = comp_s / (h2d_s > 0 ? h2d_s : 1e-30);
+    f = f < 1.25 ? 1.25 : (f > 4.0 ? 4.0 : f);
+    double w = 1.0;
+    while (bounds.back() < num_pairs) {
       const int64_t left = num_pairs - bounds.back();
-      // fold a short remainder (< 1 wave) into this chunk
-      const int64_t take = left <= (w + 1) * wave_pairs ? left : w * wave_pairs;
+      const int64_t wi = int64_t(w) > 0 ? int64_t(w) : 1;
+      // fold a remainder shorter than the next chunk into this one
+      const int64_t take = left <= int64_t(double(wi) * (1.0 + f)) * wave_pairs ? left
+                                                                                : wi * wave_pairs;
       bounds.push_back(bounds.back() + take);
+      w *= f;
     }
   }
   const int64_t nch = int64_t(bounds.size()) - 1;
