@@ -122,6 +122,191 @@ __device__ __noinline__ uint3 gather_straddle(const uint8_t* traw, int64_t tstri
 }
 
 // ---------------------------------------------------------------------------
+// Per-lane state and the wavefront step of the fused single-warp sweeps
+// (sw_sweep_kernel and sw_sweep_wrap_kernel share it).
+//
+// A lane owns query rows [sl R, sl R + R) of its segment's current group:
+// their scores at the previous column (H, R x S planes), the up-row score of
+// the previous column (dtop, the diagonal input of its first row), its
+// running max (M) or threshold flag, its query bases (xh / xl), and the
+// countdown to its next group switch.  All of it lives in registers.
+template <int S, int R, int L, int CIRC, bool PAD, class K>
+struct FusedLane {
+  static constexpr int kMW = BPBC_MODE == kModeThreshold ? L : L * S;  // Mpart words per lane-group
+  uint32_t H[R][S], dtop[S], M[S];
+  uint32_t xh[R], xl[R], kill[R];
+  uint32_t nz, z0;    // 0/1 multiplier of the received up-row; 0 (state reset on the FMA pipe)
+  uint32_t flag;      // threshold mode: pairs with a cell > tau so far
+  int cnt;            // steps until my next group starts (J % n == 0)
+  int gi;             // my current group within the (sub-)stream
+  int gsn;            // group ends stored in this (sub-)stream
+  uint32_t* mdst;     // my partial-max slot of the current group, advanced at every switch
+  const uint2* xrow;  // my query-plane slot 0 in the shared ring (+ slot * 32 * R)
+
+  __device__ __forceinline__ void reset(int sl) {
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      dtop[i] = 0;
+      M[i] = 0;
+#pragma unroll
+      for (int r = 0; r < R; ++r) H[r][i] = 0;
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
+    flag = 0;
+    cnt = sl;
+    gi = -1;
+  }
+
+  // One wavefront step with target planes y of my current column.  SW: the
+  // step may be a lane's group switch (the warp runs phases in which no lane
+  // switches without the per-step check): kSwBranch takes the switch in a
+  // divergent branch, kSwPred runs it branch-free in every lane (predicated
+  // stores and loads, state reset by a multiply with 0/1 on the FMA pipe), so
+  // the two steps of an iteration stay one basic block the scheduler can
+  // interleave.
+  template <int SW>
+  __device__ __forceinline__ void step(const uint2 y, const SweepArgs& a, const K& k) {
+    uint32_t up[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
+
+    if constexpr (SW == kSwPred) {
+      // keep = 0 at column 0 of my next group, else 1: the carry of
+      // cnt + (2^31 - 1) into bit 31, taken as mul.hi so it stays on the FMA
+      // pipe and ptxas cannot turn the resets below into selects
+      const uint32_t keep = mul_hi(uint32_t(cnt) + 0x7FFFFFFFu, 2u);
+      const bool sw = cnt == 0;
+      const uint32_t st = (sw && unsigned(gi) < unsigned(gsn)) ? 1u : 0u;
+      if constexpr (BPBC_MODE == kModeThreshold) {
+        st_if(mdst, flag, st);
+      } else {
+#pragma unroll
+        for (int i = 0; i < S; ++i) st_if(mdst + i, M[i], st);
+      }
+      mdst += st * kMW;
+      gi += sw ? 1 : 0;
+      flag = mul_lo(flag, keep);
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        M[i] = mul_lo(M[i], keep);
+        dtop[i] = mul_lo(dtop[i], keep);
+#pragma unroll
+        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], keep);
+      }
+      const uint2* xv = xrow + (gi & 1) * (32 * R);
+#pragma unroll
+      for (int r = 0; r < R; ++r) lds2_if(xv + r, xh[r], xl[r], sw ? 1u : 0u);
+      cnt = (sw ? a.n : cnt) - 1;
+    }
+    if (SW == kSwBranch && cnt == 0) {  // column 0 of my next group (divergent, once per group)
+      if (gi >= 0 && gi < gsn) {
+        if constexpr (BPBC_MODE == kModeThreshold) {
+          *mdst = flag;  // one flag word per lane
+        } else {
+          // exact circuit: M tracked D' = diag + w + g; extract subtracts g
+#pragma unroll
+          for (int i = 0; i < S; ++i) mdst[i] = M[i];
+        }
+        mdst += kMW;
+      }
+      ++gi;
+      flag = mul_lo(flag, z0);
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        M[i] = mul_lo(M[i], z0);
+        dtop[i] = mul_lo(dtop[i], z0);
+#pragma unroll
+        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], z0);
+      }
+      const uint2* xv = xrow + (gi & 1) * (32 * R);
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const uint2 v = xv[r];
+        xh[r] = v.x;
+        xl[r] = v.y;
+      }
+      cnt = a.n;
+    }
+    if (SW == kSwBranch) --cnt;
+
+    uint32_t dg[S], u[S];
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      dg[i] = dtop[i];
+      u[i] = up[i];
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      uint32_t hn[S], dn[S];
+      // running max over the diagonal term (circuit.cuh finish_exact); padded
+      // rows are masked out of it
+      if constexpr (CIRC == kExact) {
+        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn, k);
+      } else {
+        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
+      }
+      if constexpr (BPBC_MODE == kModeThreshold) {
+        flag_gt<S, PAD>(flag, dn, a.tmask, kill[r]);
+      } else {
+        runmax<S, PAD>(M, dn, kill[r]);
+      }
+#pragma unroll
+      for (int i = 0; i < S; ++i) {
+        dg[i] = H[r][i];
+        H[r][i] = hn[i];
+        u[i] = hn[i];
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < S; ++i) dtop[i] = up[i];
+  }
+
+  // The 32 steps of one phase; yb = my 32 target columns of the phase in the
+  // shared ring.  A lane switches groups in this phase iff its countdown is
+  // below 32.  Two copies of the step must fit the instruction cache together
+  // (4 warps per SMSP run both): at R = 8 one copy is ~27 KB and two copies
+  // measured 16 % slower (C3), so R = 8 keeps only the checked step.  Switch
+  // steps run branch-free (kSwPred: C2 5 743 vs 5 643 GCUPS with the
+  // divergent branch); the single R = 8 step runs in every phase and keeps
+  // the branch (kSwPred there costs every step: C3 5 194 vs 5 429).
+  //
+  // R <= 4: one loop for every phase, whose iterations (two steps each) run
+  // the switch copy only inside the phase's switch window [lo, hi] -- the
+  // steps at which some lane of the warp reaches column 0 of its next group
+  // (warp-uniform, two redux votes per phase).  The L lanes of a segment
+  // switch at L consecutive steps, so with L = 16 at most half of a phase
+  // runs the switch copy (m <= 64, where every phase or every other one has
+  // switches); with L = 32 a switch phase is switch steps throughout.
+  __device__ __forceinline__ void phase(const uint2* yb, const SweepArgs& a, const K& k) {
+    if constexpr (R > 4) {
+#pragma unroll 1
+      for (int i = 0; i < 32; i += 2) {
+        const uint2 y0 = yb[i], y1 = yb[i + 1];
+        step<kSwBranch>(y0, a, k);
+        step<kSwBranch>(y1, a, k);
+      }
+    } else {
+      // (broadcast from lane 0 so the window test runs on the uniform datapath)
+      const int lo = __shfl_sync(0xFFFFFFFFu, int(__reduce_min_sync(0xFFFFFFFFu, cnt < 32 ? unsigned(cnt) : 32u)), 0);
+      const int hi = __shfl_sync(0xFFFFFFFFu, int(__reduce_max_sync(0xFFFFFFFFu, cnt < 32 ? unsigned(cnt) + 1 : 0u)), 0) - 1;
+#pragma unroll 1
+      for (int i = 0; i < 32; i += 2) {
+        const uint2 y0 = yb[i], y1 = yb[i + 1];
+        if (i + 1 >= lo && i <= hi) {
+          step<BPBC_SWMODE>(y0, a, k);
+          step<BPBC_SWMODE>(y1, a, k);
+        } else {
+          step<kSwNone>(y0, a, k);
+          step<kSwNone>(y1, a, k);
+          cnt -= 2;
+        }
+      }
+    }
+  }
+};
+
+// ---------------------------------------------------------------------------
 // The single-warp sweep with the W2B transpose fused in:
 // it reads the caller's raw codes (u8, or 2-bit packed) and builds the bit
 // planes itself, so no separate pack pass and no planes in HBM.
@@ -146,7 +331,6 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   const int wib = threadIdx.x >> 5;
   const int64_t warp = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   if (warp * SEGS >= a.streams) return;  // uniform per warp
-  const int64_t stream = warp * SEGS + seg;
 
   // groups of segment s's stream (uniform per warp for each s)
   auto seg_range = [&](int s, int64_t& gbs, int64_t& gss) {
@@ -160,23 +344,15 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   };
   int64_t Gs, gb;
   seg_range(seg, gb, Gs);
-  const uint32_t nz = opaque(sl != 0 ? 1u : 0u);
+  FusedLane<S, R, L, CIRC, PAD, K> ln;
+  ln.nz = opaque(sl != 0 ? 1u : 0u);
   // multiplier 0 for the state reset at a group switch: the reset runs as
   // IMADs on the FMA pipe instead of register-pair clears on the ALU pipe,
   // which the cell circuits saturate
-  const uint32_t z0 = opaque(uint32_t(a.m) >> 31);  // 0 (m > 0), unknown to ptxas
-  uint32_t kill[R];
+  ln.z0 = opaque(uint32_t(a.m) >> 31);  // 0 (m > 0), unknown to ptxas
 #pragma unroll
-  for (int r = 0; r < R; ++r) kill[r] = PAD ? opaque((sl * R + r >= a.m) ? 0xFFFFFFFFu : 0u) : 0u;
-
-  uint32_t H[R][S], dtop[S], M[S];
-#pragma unroll
-  for (int i = 0; i < S; ++i) {
-    dtop[i] = 0;
-    M[i] = 0;
-#pragma unroll
-    for (int r = 0; r < R; ++r) H[r][i] = 0;
-  }
+  for (int r = 0; r < R; ++r) ln.kill[r] = PAD ? opaque((sl * R + r >= a.m) ? 0xFFFFFFFFu : 0u) : 0u;
+  ln.reset(sl);
   __shared__ uint2 xring[4][2][32][R];        // [warp][slot][lane][row]
   __shared__ uint2 yring[4][SEGS][256];       // [warp][segment][column slot, doubled]
   uint2 (*xr)[32][R] = xring[wib];
@@ -226,120 +402,9 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     }
   };
 
-  uint32_t xh[R], xl[R];
-#pragma unroll
-  for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
-  int cnt = sl;      // steps until my next group starts (J % n == 0)
-  int gi = -1;       // my current group within the stream
-  uint32_t flag = 0; // threshold mode: pairs with a cell > tau so far
-  const int gsn = int(Gs);  // groups of my stream (< 2^31: P < 2^36)
-  // my partial-max slot of the current group, advanced at every switch
-  constexpr int kMW = BPBC_MODE == kModeThreshold ? L : L * S;
-  uint32_t* mdst = a.Mpart + (gb * L + sl) * (kMW / L);
-  const uint2* xrow = &xr[0][lane][0];  // + slot * 32 * R
-
-  // One wavefront step with target planes y of my current column.  SW: the
-  // step may be a lane's group switch (the warp runs phases in which no lane
-  // switches without the per-step check): kSwBranch takes the switch in a
-  // divergent branch, kSwPred runs it branch-free in every lane (predicated
-  // stores and loads, state reset by a multiply with 0/1 on the FMA pipe), so
-  // the two steps of an iteration stay one basic block the scheduler can
-  // interleave.
-  auto step = [&](const uint2 y, auto SW) {
-    uint32_t up[S];
-#pragma unroll
-    for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
-
-    if constexpr (decltype(SW)::value == kSwPred) {
-      // keep = 0 at column 0 of my next group, else 1: the carry of
-      // cnt + (2^31 - 1) into bit 31, taken as mul.hi so it stays on the FMA
-      // pipe and ptxas cannot turn the resets below into selects
-      const uint32_t keep = mul_hi(uint32_t(cnt) + 0x7FFFFFFFu, 2u);
-      const bool sw = cnt == 0;
-      const uint32_t st = (sw && unsigned(gi) < unsigned(gsn)) ? 1u : 0u;
-      if constexpr (BPBC_MODE == kModeThreshold) {
-        st_if(mdst, flag, st);
-      } else {
-#pragma unroll
-        for (int i = 0; i < S; ++i) st_if(mdst + i, M[i], st);
-      }
-      mdst += st * kMW;
-      gi += sw ? 1 : 0;
-      flag = mul_lo(flag, keep);
-#pragma unroll
-      for (int i = 0; i < S; ++i) {
-        M[i] = mul_lo(M[i], keep);
-        dtop[i] = mul_lo(dtop[i], keep);
-#pragma unroll
-        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], keep);
-      }
-      const uint2* xv = xrow + (gi & 1) * (32 * R);
-#pragma unroll
-      for (int r = 0; r < R; ++r) lds2_if(xv + r, xh[r], xl[r], sw ? 1u : 0u);
-      cnt = (sw ? a.n : cnt) - 1;
-    }
-    if (decltype(SW)::value == kSwBranch && cnt == 0) {  // column 0 of my next group (divergent, once per group)
-      if (gi >= 0 && gi < gsn) {
-        if constexpr (BPBC_MODE == kModeThreshold) {
-          *mdst = flag;  // one flag word per lane
-        } else {
-          // exact circuit: M tracked D' = diag + w + g; extract subtracts g
-#pragma unroll
-          for (int i = 0; i < S; ++i) mdst[i] = M[i];
-        }
-        mdst += kMW;
-      }
-      ++gi;
-      flag = mul_lo(flag, z0);
-#pragma unroll
-      for (int i = 0; i < S; ++i) {
-        M[i] = mul_lo(M[i], z0);
-        dtop[i] = mul_lo(dtop[i], z0);
-#pragma unroll
-        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], z0);
-      }
-      const uint2* xv = xrow + (gi & 1) * (32 * R);
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        const uint2 v = xv[r];
-        xh[r] = v.x;
-        xl[r] = v.y;
-      }
-      cnt = a.n;
-    }
-    if (decltype(SW)::value == kSwBranch) --cnt;
-
-    uint32_t dg[S], u[S];
-#pragma unroll
-    for (int i = 0; i < S; ++i) {
-      dg[i] = dtop[i];
-      u[i] = up[i];
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      uint32_t hn[S], dn[S];
-      // running max over the diagonal term (circuit.cuh finish_exact); padded
-      // rows are masked out of it
-      if constexpr (CIRC == kExact) {
-        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn, k);
-      } else {
-        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
-      }
-      if constexpr (BPBC_MODE == kModeThreshold) {
-        flag_gt<S, PAD>(flag, dn, a.tmask, kill[r]);
-      } else {
-        runmax<S, PAD>(M, dn, kill[r]);
-      }
-#pragma unroll
-      for (int i = 0; i < S; ++i) {
-        dg[i] = H[r][i];
-        H[r][i] = hn[i];
-        u[i] = hn[i];
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < S; ++i) dtop[i] = up[i];
-  };
+  ln.gsn = int(Gs);  // groups of my stream (< 2^31: P < 2^36)
+  ln.mdst = a.Mpart + (gb * L + sl) * (ln.kMW / L);
+  ln.xrow = &xr[0][lane][0];
 
   // prologue: the first group's query planes, target chunks -1 (zeros), 0, 1
 #pragma unroll
@@ -372,31 +437,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
       }
     }
     __syncwarp();
-    const uint2* yb = &yr[seg][(32 * p - sl) & 127];  // my 32 columns of this phase
-    // a lane switches groups in this phase iff its countdown is below 32.
-    // Two copies of the loop body must fit the instruction cache together
-    // (4 warps per SMSP run both): at R = 8 one copy is ~27 KB and two copies
-    // measured 16 % slower (C3), so R = 8 keeps only the checked loop.
-    // Switch phases run branch-free (kSwPred: C2 5 743 vs 5 643 GCUPS with the
-    // divergent branch); the single R = 8 loop runs in every phase and keeps
-    // the branch (kSwPred there costs every step: C3 5 194 vs 5 429).
-    constexpr int kSw = R > 4 ? kSwBranch : BPBC_SWMODE;
-    if (R > 4 || __any_sync(0xFFFFFFFFu, cnt < 32)) {
-#pragma unroll 1
-      for (int i = 0; i < 32; i += 2) {
-        const uint2 y0 = yb[i], y1 = yb[i + 1];
-        step(y0, SwMode<kSw>{});
-        step(y1, SwMode<kSw>{});
-      }
-    } else {
-#pragma unroll 1
-      for (int i = 0; i < 32; i += 2) {
-        const uint2 y0 = yb[i], y1 = yb[i + 1];
-        step(y0, SwMode<kSwNone>{});
-        step(y1, SwMode<kSwNone>{});
-      }
-      cnt -= 32;
-    }
+    ln.phase(&yr[seg][(32 * p - sl) & 127], a, k);  // my 32 columns of this phase
   }
   if (__any_sync(0xFFFFFFFFu, bad != 0) && lane == 0) atomicOr(a.flags, BPBC_FLAG_BAD_BASE);
 }
@@ -429,75 +470,57 @@ __device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
 }
 
 
-template <int S, int R, int CIRC, bool PAD, class K>
 // (no occupancy floor: the schedule runs it with few blocks per SM; the
 // planner reads its occupancy)
+template <int S, int R, int CIRC, bool PAD, class K>
 __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, const K k) {
-  constexpr int L = 32, SEGS = 1;
+  constexpr int L = 32;
   constexpr int XCH = (L * R + 31) / 32;  // 32-row chunks of a group's query rows
   constexpr int NSW = snap_words(R, S);
   const int lane = threadIdx.x & 31;
-  const int sl = lane & (L - 1);
-  const int seg = lane / L;
   // warp index broadcast from lane 0: provably warp-uniform, so the
   // sub-stream bookkeeping derived from it stays on the uniform datapath
   const int wib = __shfl_sync(0xFFFFFFFFu, int(threadIdx.x >> 5), 0);
   const int64_t warp = int64_t(blockIdx.x) * (blockDim.x >> 5) + wib;
-  if (warp * SEGS >= a.streams) return;  // uniform per warp
+  if (warp >= a.streams) return;  // uniform per warp
 
-  const uint32_t nz = opaque(sl != 0 ? 1u : 0u);
-  // multiplier 0 for the state reset at a group switch: the reset runs as
-  // IMADs on the FMA pipe instead of register-pair clears on the ALU pipe,
-  // which the cell circuits saturate
-  const uint32_t z0 = opaque(uint32_t(a.m) >> 31);  // 0 (m > 0), unknown to ptxas
-  uint32_t kill[R];
+  FusedLane<S, R, L, CIRC, PAD, K> ln;
+  ln.nz = opaque(lane != 0 ? 1u : 0u);
+  ln.z0 = opaque(uint32_t(a.m) >> 31);  // 0 (m > 0), unknown to ptxas
 #pragma unroll
-  for (int r = 0; r < R; ++r) kill[r] = PAD ? opaque((sl * R + r >= a.m) ? 0xFFFFFFFFu : 0u) : 0u;
-
-  uint32_t H[R][S], dtop[S], M[S];
-  __shared__ uint2 xring[4][2][32][R];        // [warp][slot][lane][row]
-  __shared__ uint2 yring[4][SEGS][256];       // [warp][segment][column slot, doubled]
+  for (int r = 0; r < R; ++r) ln.kill[r] = PAD ? opaque((lane * R + r >= a.m) ? 0xFFFFFFFFu : 0u) : 0u;
+  __shared__ uint2 xring[4][2][32][R];  // [warp][slot][lane][row]
+  __shared__ uint2 yring[4][256];       // [warp][column slot, doubled]
   uint2 (*xr)[32][R] = xring[wib];
-  uint2 (*yr)[256] = yring[wib];
+  uint2* yr = yring[wib];
+  ln.xrow = &xr[0][lane][0];
   const bool packed2 = a.packed2 != 0;
   const int mypos = packed2 ? tr_pos_packed2(lane) : tr_pos_u8(lane);
   uint32_t bad = 0;
 
-  // Sub-stream bookkeeping per segment (uniform per segment): first group,
-  // groups touched, the next target chunk's (group offset, column) and the
-  // next query group with the step from which it may be built.
-  int64_t g0[SEGS], nspan[SEGS], yg[SEGS], xnext[SEGS], xth[SEGS];
-  int ycol[SEGS];
-
-  // the next 32 target columns of segment s -> ring chunk c; advance
-  auto build_y = [&](int s, int64_t c) {
+  // sub-stream bookkeeping (warp-uniform): first group g0, groups touched
+  // nspan, the next target chunk (group offset yg, column ycol) and the next
+  // query group xnext with the step xth from which it may be built
+  int64_t g0 = 0, nspan = 0, yg = 0, xnext = 0, xth = 0;
+  int ycol = 0;
+  // the next 32 target columns -> ring chunk c; advance (n % 32 == 0 here)
+  auto build_y = [&](int64_t c) {
     uint32_t Hw = 0, Lw = 0;
-    if (yg[s] < nspan[s]) {
-      const int64_t g = g0[s] + yg[s];
-      const int col = ycol[s];
-      if (col + 32 <= a.n) {
-        tr_load_fold(a.traw, a.tstride, a.n, g * 32 + lane, a.P, col, packed2, Hw, Lw, bad);
-      } else {  // the chunk straddles two groups (n % 32 != 0; n >= 48)
-        const uint3 r3 = gather_straddle(a.traw, a.tstride, a.n, a.P, g, yg[s] + 1 < nspan[s],
-                                         col, lane, packed2);
-        Hw = r3.x;
-        Lw = r3.y;
-        bad |= r3.z;
-      }
-    }
+    if (yg < nspan)
+      tr_load_fold(a.traw, a.tstride, a.n, (g0 + yg) * 32 + lane, a.P, ycol, packed2, Hw, Lw, bad);
     tr_butterfly(Hw, Lw, lane);
     const int slot = int((32 * c + mypos) & 127);
-    yr[s][slot] = make_uint2(Hw, Lw);
-    yr[s][slot + 128] = make_uint2(Hw, Lw);
-    ycol[s] += 32;
-    if (ycol[s] >= a.n) {  // (n >= 32 on this kernel)
-      ycol[s] -= a.n;
-      ++yg[s];
+    yr[slot] = make_uint2(Hw, Lw);
+    yr[slot + 128] = make_uint2(Hw, Lw);
+    ycol += 32;
+    if (ycol >= a.n) {
+      ycol -= a.n;
+      ++yg;
     }
   };
-  // query rows of segment s's group h (sub-stream-relative) -> x slot h & 1
-  auto build_x = [&](int s, int64_t h) {
-    int64_t g = g0[s] + h;
+  // query rows of group g0 + h -> x slot h & 1
+  auto build_x = [&](int64_t h) {
+    int64_t g = g0 + h;
     g = g < a.G ? g : a.G - 1;
 #pragma unroll
     for (int c = 0; c < XCH; ++c) {
@@ -505,200 +528,67 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
       tr_load_fold(a.qraw, a.qstride, a.m, g * 32 + lane, a.P, 32 * c, packed2, Hw, Lw, bad);
       tr_butterfly(Hw, Lw, lane);
       const int row = 32 * c + mypos;  // rows >= m are zero (tr_load_fold)
-      if (row < L * R) xr[int(h & 1)][s * L + row / R][row % R] = make_uint2(Hw, Lw);
+      if (row < L * R) xr[int(h & 1)][row / R][row % R] = make_uint2(Hw, Lw);
     }
   };
 
-  uint32_t xh[R], xl[R];
-  int cnt = 0;       // steps until my next group starts (J % n == 0)
-  int gi = -1;       // my current group within the sub-stream
-  uint32_t flag = 0; // threshold mode: pairs with a cell > tau so far
-  int gsn = 0;       // group ends my segment stores in this sub-stream
-  // my partial-max slot of the current group, advanced at every switch
-  constexpr int kMW = BPBC_MODE == kModeThreshold ? L : L * S;
-  uint32_t* mdst = a.Mpart;
-  const uint2* xrow = &xr[0][lane][0];  // + slot * 32 * R
-
-  // One wavefront step with target planes y of my current column.  SW: the
-  // step may be a lane's group switch (the warp runs phases in which no lane
-  // switches without the per-step check): kSwBranch takes the switch in a
-  // divergent branch, kSwPred runs it branch-free in every lane (predicated
-  // stores and loads, state reset by a multiply with 0/1 on the FMA pipe), so
-  // the two steps of an iteration stay one basic block the scheduler can
-  // interleave.
-  auto step = [&](const uint2 y, auto SW) {
-    uint32_t up[S];
-#pragma unroll
-    for (int i = 0; i < S; ++i) up[i] = mul_lo(__shfl_up_sync(0xFFFFFFFFu, H[R - 1][i], 1, L), nz);
-
-    if constexpr (decltype(SW)::value == kSwPred) {
-      // keep = 0 at column 0 of my next group, else 1: the carry of
-      // cnt + (2^31 - 1) into bit 31, taken as mul.hi so it stays on the FMA
-      // pipe and ptxas cannot turn the resets below into selects
-      const uint32_t keep = mul_hi(uint32_t(cnt) + 0x7FFFFFFFu, 2u);
-      const bool sw = cnt == 0;
-      const uint32_t st = (sw && unsigned(gi) < unsigned(gsn)) ? 1u : 0u;
-      if constexpr (BPBC_MODE == kModeThreshold) {
-        st_if(mdst, flag, st);
-      } else {
-#pragma unroll
-        for (int i = 0; i < S; ++i) st_if(mdst + i, M[i], st);
-      }
-      mdst += st * kMW;
-      gi += sw ? 1 : 0;
-      flag = mul_lo(flag, keep);
-#pragma unroll
-      for (int i = 0; i < S; ++i) {
-        M[i] = mul_lo(M[i], keep);
-        dtop[i] = mul_lo(dtop[i], keep);
-#pragma unroll
-        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], keep);
-      }
-      const uint2* xv = xrow + (gi & 1) * (32 * R);
-#pragma unroll
-      for (int r = 0; r < R; ++r) lds2_if(xv + r, xh[r], xl[r], sw ? 1u : 0u);
-      cnt = (sw ? a.n : cnt) - 1;
-    }
-    if (decltype(SW)::value == kSwBranch && cnt == 0) {  // column 0 of my next group (divergent, once per group)
-      if (gi >= 0 && gi < gsn) {
-        if constexpr (BPBC_MODE == kModeThreshold) {
-          *mdst = flag;  // one flag word per lane
-        } else {
-          // exact circuit: M tracked D' = diag + w + g; extract subtracts g
-#pragma unroll
-          for (int i = 0; i < S; ++i) mdst[i] = M[i];
-        }
-        mdst += kMW;
-      }
-      ++gi;
-      flag = mul_lo(flag, z0);
-#pragma unroll
-      for (int i = 0; i < S; ++i) {
-        M[i] = mul_lo(M[i], z0);
-        dtop[i] = mul_lo(dtop[i], z0);
-#pragma unroll
-        for (int r = 0; r < R; ++r) H[r][i] = mul_lo(H[r][i], z0);
-      }
-      const uint2* xv = xrow + (gi & 1) * (32 * R);
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        const uint2 v = xv[r];
-        xh[r] = v.x;
-        xl[r] = v.y;
-      }
-      cnt = a.n;
-    }
-    if (decltype(SW)::value == kSwBranch) --cnt;
-
-    uint32_t dg[S], u[S];
-#pragma unroll
-    for (int i = 0; i < S; ++i) {
-      dg[i] = dtop[i];
-      u[i] = up[i];
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      uint32_t hn[S], dn[S];
-      // running max over the diagonal term (circuit.cuh finish_exact); padded
-      // rows are masked out of it
-      if constexpr (CIRC == kExact) {
-        cell_exact<S, K, false>(u, H[r], dg, xh[r], xl[r], y.x, y.y, 0u, hn, dn, k);
-      } else {
-        cell_sat<S, K>(u, H[r], dg, xh[r], xl[r], y.x, y.y, hn, dn, k);
-      }
-      if constexpr (BPBC_MODE == kModeThreshold) {
-        flag_gt<S, PAD>(flag, dn, a.tmask, kill[r]);
-      } else {
-        runmax<S, PAD>(M, dn, kill[r]);
-      }
-#pragma unroll
-      for (int i = 0; i < S; ++i) {
-        dg[i] = H[r][i];
-        H[r][i] = hn[i];
-        u[i] = hn[i];
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < S; ++i) dtop[i] = up[i];
-  };
-
+  const int64_t tot = a.G * a.n;
+  const int64_t V0 = warp * a.span;
+  const int64_t V1 = V0 + a.span < tot ? V0 + a.span : tot;
+  const int64_t ga = V0 / a.n, gz = V1 / a.n;
+  const int ra = int(V0 - ga * a.n), rb = int(V1 - gz * a.n);
 #pragma unroll 1
   for (int sub = 0; sub < 3; ++sub) {
     // ---- this sub-stream's groups, first column and boundary behaviour
-    int c0 = 0;                       // first column (of group g0)
+    int c0 = 0;  // first column (of group g0)
     bool snap_in = false, snap_out = false;
-    int64_t steps = 0, slot = 0, mygs = 0;
-    {
-      const int64_t tot = a.G * a.n;
-      const int64_t V0 = warp * a.span;
-      const int64_t V1 = V0 + a.span < tot ? V0 + a.span : tot;
-      const int64_t ga = V0 / a.n, gz = V1 / a.n;
-      const int ra = int(V0 - ga * a.n), rb = int(V1 - gz * a.n);
-      if (sub == 0) {  // head of group gz: columns [0, rb), snapshot out
-        if (rb == 0) continue;
-        g0[0] = gz;
-        nspan[0] = 1;
-        snap_out = true;
-        slot = warp + 1;
-        steps = rb;  // (a multiple of 32)
-      } else if (sub == 1) {  // whole groups
-        g0[0] = ga + (ra > 0 ? 1 : 0);
-        nspan[0] = gz - g0[0];
-        if (nspan[0] <= 0) continue;
-        mygs = nspan[0];
-        steps = (nspan[0] * a.n + L + 31) / 32 * 32;
-      } else {  // tail of group ga: columns [ra, n), snapshot in
-        if (ra == 0) continue;
-        g0[0] = ga;
-        nspan[0] = 1;
-        mygs = 1;
-        c0 = ra;
-        snap_in = true;
-        slot = warp;
-        steps = (a.n - ra + L + 31) / 32 * 32;
-      }
+    int64_t steps = 0, slot = 0;
+    int gs = 0;  // group ends stored
+    if (sub == 0) {  // head of group gz: columns [0, rb), snapshot out
+      if (rb == 0) continue;
+      g0 = gz;
+      nspan = 1;
+      snap_out = true;
+      slot = warp + 1;
+      steps = rb;  // (a multiple of 32)
+    } else if (sub == 1) {  // whole groups
+      g0 = ga + (ra > 0 ? 1 : 0);
+      nspan = gz - g0;
+      if (nspan <= 0) continue;
+      gs = int(nspan);
+      steps = (nspan * a.n + L + 31) / 32 * 32;
+    } else {  // tail of group ga: columns [ra, n), snapshot in
+      if (ra == 0) continue;
+      g0 = ga;
+      nspan = 1;
+      gs = 1;
+      c0 = ra;
+      snap_in = true;
+      slot = warp;
+      steps = (a.n - ra + L + 31) / 32 * 32;
     }
-
     // ---- fresh state (a lane enters its first group at its switch step)
-#pragma unroll
-    for (int i = 0; i < S; ++i) {
-      dtop[i] = 0;
-      M[i] = 0;
-#pragma unroll
-      for (int r = 0; r < R; ++r) H[r][i] = 0;
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r) xh[r] = xl[r] = 0;
-    flag = 0;
-    cnt = sl;
-    gi = -1;
-    gsn = int(mygs);
-    mdst = a.Mpart + (g0[seg] * L + sl) * (kMW / L);
+    ln.reset(lane);
+    ln.gsn = gs;
+    ln.mdst = a.Mpart + (g0 * L + lane) * (ln.kMW / L);
 
     // ---- prologue: first group's query planes, target chunks -1 (zeros, or
     // the columns before c0 when resuming), 0, 1
     __syncwarp();  // the previous sub-stream's ring reads -> these writes
-#pragma unroll
-    for (int s = 0; s < SEGS; ++s) {
-      yr[s][lane] = yr[s][lane + 32] = yr[s][lane + 64] = yr[s][lane + 96] = make_uint2(0u, 0u);
-      yr[s][lane + 128] = yr[s][lane + 160] = yr[s][lane + 192] = yr[s][lane + 224] =
-          make_uint2(0u, 0u);
-    }
+    yr[lane] = yr[lane + 32] = yr[lane + 64] = yr[lane + 96] = make_uint2(0u, 0u);
+    yr[lane + 128] = yr[lane + 160] = yr[lane + 192] = yr[lane + 224] = make_uint2(0u, 0u);
     __syncwarp();
-#pragma unroll
-    for (int s = 0; s < SEGS; ++s) {
-      xnext[s] = 1;
-      xth[s] = L - c0;  // group h may be built once (h-1) n - c0 + L <= 32 p
-      build_x(s, 0);
-      yg[s] = 0;
-      ycol[s] = c0;
-      if (snap_in) {
-        ycol[s] = c0 - 32;  // (c0 >= 32)
-        build_y(s, -1);
-      }
-      build_y(s, 0);
-      build_y(s, 1);
+    xnext = 1;
+    xth = L - c0;  // group h may be built once (h-1) n - c0 + L <= 32 p
+    build_x(0);
+    yg = 0;
+    ycol = c0;
+    if (snap_in) {
+      ycol = c0 - 32;  // (c0 >= 32)
+      build_y(-1);
     }
+    build_y(0);
+    build_y(1);
     if (snap_in) {  // resume the warp state the previous stream left at column c0
       // (every lane polls; the vote keeps the loop warp-uniform)
       while (__any_sync(0xFFFFFFFFu, ld_acquire_gpu(a.snap_flag + slot) == 0)) __nanosleep(256);
@@ -706,72 +596,45 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
 #pragma unroll
       for (int i = 0; i < S; ++i) {
 #pragma unroll
-        for (int r = 0; r < R; ++r) H[r][i] = __ldcg(src + (r * S + i) * 32);
-        dtop[i] = __ldcg(src + (R * S + i) * 32);
-        if constexpr (BPBC_MODE != kModeThreshold) M[i] = __ldcg(src + ((R + 1) * S + i) * 32);
+        for (int r = 0; r < R; ++r) ln.H[r][i] = __ldcg(src + (r * S + i) * 32);
+        ln.dtop[i] = __ldcg(src + (R * S + i) * 32);
+        if constexpr (BPBC_MODE != kModeThreshold) ln.M[i] = __ldcg(src + ((R + 1) * S + i) * 32);
       }
-      if constexpr (BPBC_MODE == kModeThreshold) flag = __ldcg(src + (R + 1) * S * 32);
-      cnt = int(a.n - c0) + sl;
-      gi = 0;
+      if constexpr (BPBC_MODE == kModeThreshold) ln.flag = __ldcg(src + (R + 1) * S * 32);
+      ln.cnt = int(a.n - c0) + lane;
+      ln.gi = 0;
 #pragma unroll
       for (int r = 0; r < R; ++r) {  // (slot 0, written by build_x above)
-        const uint2 v = xrow[r];
-        xh[r] = v.x;
-        xl[r] = v.y;
+        const uint2 v = ln.xrow[r];
+        ln.xh[r] = v.x;
+        ln.xl[r] = v.y;
       }
     }
 
     const int64_t phases = steps / 32;  // steps is a multiple of 32
     for (int64_t p = 0; p < phases; ++p) {
       __syncwarp();  // this warp's ring writes of the previous phase -> reads
-#pragma unroll
-      for (int s = 0; s < SEGS; ++s) {
-        build_y(s, p + 2);
-        // group h's query may be written into slot h & 1 once every lane of
-        // the segment has entered group h - 1; lane 0 needs it at its start
-        if (xth[s] <= 32 * p) {
-          build_x(s, xnext[s]);
-          ++xnext[s];
-          xth[s] += a.n;
-        }
+      build_y(p + 2);
+      // group h's query may be written into slot h & 1 once every lane has
+      // entered group h - 1; lane 0 needs it at its start
+      if (xth <= 32 * p) {
+        build_x(xnext);
+        ++xnext;
+        xth += a.n;
       }
       __syncwarp();
-      const uint2* yb = &yr[seg][(32 * p - sl) & 127];  // my 32 columns of this phase
-      // a lane switches groups in this phase iff its countdown is below 32.
-      // Two copies of the loop body must fit the instruction cache together
-      // (4 warps per SMSP run both): at R = 8 one copy is ~27 KB and two copies
-      // measured 16 % slower (C3), so R = 8 keeps only the checked loop.
-      // Switch phases run branch-free (kSwPred: C2 5 743 vs 5 643 GCUPS with the
-      // divergent branch); the single R = 8 loop runs in every phase and keeps
-      // the branch (kSwPred there costs every step: C3 5 194 vs 5 429).
-      constexpr int kSw = R > 4 ? kSwBranch : BPBC_SWMODE;
-      if (R > 4 || __any_sync(0xFFFFFFFFu, cnt < 32)) {
-#pragma unroll 1
-        for (int i = 0; i < 32; i += 2) {
-          const uint2 y0 = yb[i], y1 = yb[i + 1];
-          step(y0, SwMode<kSw>{});
-          step(y1, SwMode<kSw>{});
-        }
-      } else {
-#pragma unroll 1
-        for (int i = 0; i < 32; i += 2) {
-          const uint2 y0 = yb[i], y1 = yb[i + 1];
-          step(y0, SwMode<kSwNone>{});
-          step(y1, SwMode<kSwNone>{});
-        }
-        cnt -= 32;
-      }
+      ln.phase(&yr[(32 * p - lane) & 127], a, k);  // my 32 columns of this phase
     }
     if (snap_out) {  // hand the warp state to the stream that finishes this group
       uint32_t* dst = a.snap + slot * (NSW * 32) + lane;
 #pragma unroll
       for (int i = 0; i < S; ++i) {
 #pragma unroll
-        for (int r = 0; r < R; ++r) __stcg(dst + (r * S + i) * 32, H[r][i]);
-        __stcg(dst + (R * S + i) * 32, dtop[i]);
-        if constexpr (BPBC_MODE != kModeThreshold) __stcg(dst + ((R + 1) * S + i) * 32, M[i]);
+        for (int r = 0; r < R; ++r) __stcg(dst + (r * S + i) * 32, ln.H[r][i]);
+        __stcg(dst + (R * S + i) * 32, ln.dtop[i]);
+        if constexpr (BPBC_MODE != kModeThreshold) __stcg(dst + ((R + 1) * S + i) * 32, ln.M[i]);
       }
-      if constexpr (BPBC_MODE == kModeThreshold) __stcg(dst + (R + 1) * S * 32, flag);
+      if constexpr (BPBC_MODE == kModeThreshold) __stcg(dst + (R + 1) * S * 32, ln.flag);
       __threadfence();
       __syncwarp();
       if (lane == 0) st_release_gpu(a.snap_flag + slot, 1u);

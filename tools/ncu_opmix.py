@@ -8,6 +8,7 @@ the launch's word-cell count is given), split into the pipes the sweep
 cares about, plus the share of stall samples per opcode.
 """
 import csv
+import gzip
 import re
 import sys
 from collections import Counter
@@ -17,7 +18,7 @@ ALU = {"LOP3", "ISETP", "SEL", "SHF", "IADD3", "PLOP3", "LEA", "FLO", "POPC", "B
 
 
 def main():
-    rows = list(csv.reader(open(sys.argv[1])))
+    rows = list(csv.reader(gzip.open(sys.argv[1], "rt") if sys.argv[1].endswith(".gz") else open(sys.argv[1])))
     h = rows[1]
     ie = h.index("Instructions Executed")
     src = h.index("Source")

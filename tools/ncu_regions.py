@@ -7,12 +7,13 @@ usage: ncu_regions.py <source.csv> name=0xa-0xb [name=0xc-0xd ...]
 Used for the sweep kernel's fast / switch / per-phase split.
 """
 import csv
+import gzip
 import sys
 from collections import Counter, defaultdict
 
 
 def main():
-    rows = list(csv.reader(open(sys.argv[1])))
+    rows = list(csv.reader(gzip.open(sys.argv[1], "rt") if sys.argv[1].endswith(".gz") else open(sys.argv[1])))
     ranges = {}
     for arg in sys.argv[2:]:
         k, v = arg.split("=")

@@ -41,9 +41,16 @@ KEYS = [
 STALL = re.compile(r"smsp__average_warps_issue_stalled_(\w+)_per_issue_active\.ratio")
 
 
+def raw_csv(path):
+    """--page raw --csv of a report, or the exported text itself (.csv)."""
+    if path.endswith(".csv"):
+        return open(path).read()
+    return subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
+                          text=True).stdout
+
+
 def report(path):
-    raw = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
-                         text=True).stdout
+    raw = raw_csv(path)
     rows = list(csv.reader(io.StringIO(raw)))
     if len(rows) < 3:
         print(f"{path}: no data")
@@ -90,8 +97,7 @@ def launches(path):
 def record(path, key, pattern="sw_sweep"):
     import json
     import os
-    raw = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
-                         text=True).stdout
+    raw = raw_csv(path)
     rows = list(csv.reader(io.StringIO(raw)))
     hdr = rows[0]
     for r in rows[2:]:

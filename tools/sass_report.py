@@ -7,6 +7,8 @@ Theorem 6).
 
 usage: python tools/sass_report.py [--build build/csrc] [--json]
 
+The "switch-free loop" is the straight-line two-step block of the hot loop
+without the group-switch code (the switch copy runs only in switch windows).
 One word-cell = one 32-bit word of one DP cell = 32 cells.  A loop
 iteration runs two wavefront steps of R rows per lane, i.e. 2 R word-cells
 per thread, so LOP3 per word-cell = LOP3 in the loop / (2 R).
@@ -79,6 +81,31 @@ def loops(ins):
     return inner
 
 
+def basic_blocks(ins, lo, hi):
+    """Split a loop body into straight-line blocks at branches and at the
+    targets of branches inside it: [(start, end, Counter of opcodes)]."""
+    targets = set()
+    for a, t in ins:
+        m = re.search(r"BRA(?:\.\w+)*\s.*?0x([0-9a-f]+)", t)
+        if m and lo <= int(m.group(1), 16) <= hi:
+            targets.add(int(m.group(1), 16))
+    out, cur, start = [], Counter(), None
+    for a, t in ins:
+        if a in targets and cur:
+            out.append((start, prev, cur))
+            cur, start = Counter(), None
+        if start is None:
+            start = a
+        cur[opcode(t)] += 1
+        prev = a
+        if "BRA" in t:
+            out.append((start, a, cur))
+            cur, start = Counter(), None
+    if cur:
+        out.append((start, prev, cur))
+    return out
+
+
 def report(build):
     rows = []
     for label, width, pat, R, hand in HEADLINE:
@@ -90,8 +117,20 @@ def report(build):
             rows.append({"kernel": label, "error": f"{pat} not found in {obj}"})
             continue
         inner = [l for l in loops(funcs[name]) if l[2]["LOP3"] > 100]
-        # the switch-free loop = the hot loop with the fewest non-LOP3 instructions
-        best = min(inner, key=lambda l: sum(l[2].values()) - l[2]["LOP3"])
+        # straight-line blocks of the hot loops (split at branches and branch
+        # targets): the switch-free two-step body = the big block with the
+        # fewest non-LOP3 instructions
+        blocks = []
+        for lo, hi, _ in inner:
+            blocks += basic_blocks([(a_, t) for a_, t in funcs[name] if lo <= a_ <= hi], lo, hi)
+        # a candidate holds two whole steps (>= 90 % of the hand count's LOP3);
+        # loops whose steps contain a divergent switch branch (R = 8, the
+        # multi-warp kernel) are taken whole
+        need = 0.9 * 2 * R * hand
+        cands = [b_ for b_ in blocks if b_[2]["LOP3"] >= need] or \
+                [l for l in inner if l[2]["LOP3"] >= need]
+        blocks = [b_ for b_ in blocks if b_[2]["LOP3"] > 100]
+        best = min(cands, key=lambda l: sum(l[2].values()) - l[2]["LOP3"])
         total = sum(best[2].values())
         lop3 = best[2]["LOP3"]
         rows.append({"kernel": label, "symbol_pattern": pat, "loop": f"{best[0]:#x}..{best[1]:#x}",
@@ -99,7 +138,9 @@ def report(build):
                      "lop3_per_word_cell": lop3 / (2 * R), "hand_count": hand,
                      "other": {k: v for k, v in best[2].most_common() if k != "LOP3"},
                      "loops": [{"range": f"{l[0]:#x}..{l[1]:#x}", "instructions": sum(l[2].values()),
-                                "lop3": l[2]["LOP3"]} for l in inner]})
+                                "lop3": l[2]["LOP3"]} for l in inner],
+                     "blocks": [{"range": f"{b_[0]:#x}..{b_[1]:#x}", "instructions": sum(b_[2].values()),
+                                 "lop3": b_[2]["LOP3"]} for b_ in blocks]})
     return rows
 
 
@@ -112,7 +153,7 @@ def main():
     if a.json:
         print(json.dumps(rows, indent=1))
         return
-    print("| kernel | hot loop | instr / 2 steps | LOP3 / 2 steps | LOP3 per word-cell | hand count | other opcodes |")
+    print("| kernel | switch-free block | instr / 2 steps | LOP3 / 2 steps | LOP3 per word-cell | hand count | other opcodes |")
     print("|---|---|---|---|---|---|---|")
     for r in rows:
         if "error" in r:
