@@ -45,8 +45,9 @@
  *     (give concurrent streams separate workspaces);
  *   - a ctx is not thread-safe: use one ctx per device per host thread;
  *   - the environment is read once, in bpbc_sw_init (benchmark knobs only:
- *     BPBC_MAX_BLOCKS_PER_SM, BPBC_NO_EXACT_RUN, BPBC_WRAP); no call on the
- *     hot path reads it.
+ *     BPBC_MAX_BLOCKS_PER_SM, BPBC_NO_EXACT_RUN, BPBC_WRAP,
+ *     BPBC_CHUNKED_HOST, BPBC_FORCE_WIDTH -- see DESIGN.md 6.4); no call on
+ *     the hot path reads it.
  */
 #ifndef BPBC_SW_H
 #define BPBC_SW_H
@@ -150,15 +151,22 @@ int bpbc_sw_score_batch(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8_t *t
 /*
  * End-to-end variant with HOST buffers (the paper's Steps 1-5):
  * copies the inputs host->device, runs the hot path and copies the scores
- * device->host.  The batch is cut into chunks of whole waves (one 32-pair
- * group per resident sweep stream) that flow through three ctx-owned
- * buffer slots on three ctx-owned streams (copy-in, kernels, copy-out), so
- * the copy of chunk c+1 and the result copy of chunk c-1 overlap the kernels
- * of chunk c.  The chunk plan uses the H2D and cell rates this ctx measured
- * on its previous host call.  Batches with few groups (the wrap-around
- * schedule) run as one chunk.  Pinned inputs overlap (pageable ones are
- * staged by the driver); a pageable out_scores goes through pinned staging.
- * Blocking: returns when out_scores is written.
+ * device->host.  Plans of the fused single-warp kernel (min(m, n) <= 256)
+ * run as ONE streamed launch: the inputs are copied wave by wave (a wave =
+ * one 32-pair group per resident sweep stream, contiguous because the fused
+ * kernel assigns groups to streams strided) on a ctx-owned copy stream, each
+ * wave followed by a device-side progress write (cuStreamWriteValue32), while
+ * the sweep runs concurrently on the ctx's compute stream and waits for a
+ * wave's progress before reading it; only the first wave's copy is exposed.
+ * Other plans (and devices without stream memory writes) cut the batch into
+ * chunks of whole waves that flow through three ctx-owned buffer slots on
+ * three ctx-owned streams (copy-in, kernels, copy-out), so the copy of chunk
+ * c+1 and the result copy of chunk c-1 overlap the kernels of chunk c; the
+ * chunk plan uses the H2D and cell rates this ctx measured on its previous
+ * host call.  Batches with few groups (the wrap-around schedule) run as one
+ * chunk.  Pinned inputs overlap (pageable ones are staged by the driver); a
+ * pageable out_scores goes through pinned staging.  Blocking: returns when
+ * out_scores is written.
  *
  * query, target  host, uint8 [num_pairs][m] / [num_pairs][n].
  * out_scores     host, int32 [num_pairs].
@@ -280,8 +288,11 @@ int bpbc_sw_last_launches(bpbc_sw_ctx *ctx, int32_t *kernels, int32_t *fused);
  * schedule (streams take equal runs of the concatenated target columns and
  * hand split groups over as warp-state snapshots), 0 for the
  * group-granular split; blocks_per_sm = resident sweep blocks per SM the
- * plan chose.  Either pointer may be NULL. */
-int bpbc_sw_last_schedule(bpbc_sw_ctx *ctx, int32_t *wrap, int64_t *blocks_per_sm);
+ * plan chose; host_streamed = 1 if the last bpbc_sw_score_batch_host* call
+ * ran as one streamed launch (below), 0 if chunked.  Any pointer may be
+ * NULL. */
+int bpbc_sw_last_schedule(bpbc_sw_ctx *ctx, int32_t *wrap, int64_t *blocks_per_sm,
+                          int32_t *host_streamed);
 
 /* Per-phase device timing, the columns of the paper's Table IV (P:L384-413:
  * W2B, SWA, B2W).  bpbc_sw_profile(ctx, 1) clears the accumulators and makes

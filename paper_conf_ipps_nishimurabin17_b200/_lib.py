@@ -61,7 +61,8 @@ SIGNATURES = {
                                      _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int32),
                                      _c.POINTER(_c.c_int64), _c.POINTER(_c.c_int32)]),
     "bpbc_sw_last_launches": (_c.c_int, [_vp, _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int32)]),
-    "bpbc_sw_last_schedule": (_c.c_int, [_vp, _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int64)]),
+    "bpbc_sw_last_schedule": (_c.c_int, [_vp, _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int64),
+                                         _c.POINTER(_c.c_int32)]),
     "bpbc_sw_profile": (_c.c_int, [_vp, _c.c_int]),
     "bpbc_sw_profile_read": (_c.c_int, [_vp, _c.POINTER(_c.c_double), _c.POINTER(_c.c_int64)]),
     "bpbc_sw_status_string": (_c.c_char_p, [_c.c_int]),

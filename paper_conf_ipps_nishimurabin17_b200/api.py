@@ -310,12 +310,14 @@ def last_plan(device: int = 0) -> dict:
                                         ctypes.byref(o)))
     k, f = ctypes.c_int32(), ctypes.c_int32()
     check(_lib.load().bpbc_sw_last_launches(_ctx(device), ctypes.byref(k), ctypes.byref(f)))
-    wr, bps = ctypes.c_int32(), ctypes.c_int64()
-    check(_lib.load().bpbc_sw_last_schedule(_ctx(device), ctypes.byref(wr), ctypes.byref(bps)))
+    wr, bps, hs = ctypes.c_int32(), ctypes.c_int64(), ctypes.c_int32()
+    check(_lib.load().bpbc_sw_last_schedule(_ctx(device), ctypes.byref(wr), ctypes.byref(bps),
+                                            ctypes.byref(hs)))
     return {"circuit": ["exact", "saturating"][c.value] if c.value >= 0 else None,
             "width": w.value, "rows_per_lane": r.value, "lanes": l.value,
             "streams": s.value, "ops_per_word_cell": o.value, "kernels": k.value,
-            "fused": bool(f.value), "wrap": bool(wr.value), "blocks_per_sm": bps.value}
+            "fused": bool(f.value), "wrap": bool(wr.value), "blocks_per_sm": bps.value,
+            "host_streamed": bool(hs.value)}
 
 
 def profile(enable: bool, device: int = 0) -> None:

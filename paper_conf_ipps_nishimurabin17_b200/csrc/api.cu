@@ -47,6 +47,8 @@ struct bpbc_sw_ctx {
   int opt_max_blocks = 0;       // BPBC_MAX_BLOCKS_PER_SM: cap on resident sweep blocks / SM
   bool opt_no_exact_run = false;  // BPBC_NO_EXACT_RUN: exact circuit only for (+2,-1,-1)
   int opt_wrap = -1;            // BPBC_WRAP: -1 auto, 0 never, 1 whenever valid
+  bool opt_chunked_host = false;  // BPBC_CHUNKED_HOST: host path always in chunks
+  bool opt_force_width = false;   // BPBC_FORCE_WIDTH: evaluate the circuit at score_bits
   // ctx-owned device workspace (workspace == NULL; the filter's compaction
   // scratch is a section of it): stream-ordered (cudaMallocAsync / cudaFreeAsync); a call on another
   // stream waits for buf_ev, the event after the last call that used them
@@ -61,12 +63,21 @@ struct bpbc_sw_ctx {
   HostSlot slots[kHostSlots];
   int32_t* h_out = nullptr;  // pinned staging for pageable outputs
   size_t h_out_bytes = 0;
+  // streamed host path: whole-batch device inputs / scores / workspace, the
+  // wave progress word and its reset event, copy timing events
+  uint8_t* s_q = nullptr;
+  uint8_t* s_t = nullptr;
+  int32_t* s_out = nullptr;
+  void* s_ws = nullptr;
+  size_t s_q_bytes = 0, s_t_bytes = 0, s_out_bytes = 0, s_ws_bytes = 0;
+  uint32_t* progress = nullptr;
+  cudaEvent_t ev_reset = nullptr, ev_c0 = nullptr, ev_c1 = nullptr;
   double h2d_bps = 50e9;     // measured H2D bytes/s (updated after each host call)
   double cells_ps = 5e12;    // measured cell updates/s of the device path
   char err[512] = {0};
   // last plan
   int32_t plan_circuit = -1, plan_width = 0, plan_R = 0, plan_L = 0, plan_ops = 0;
-  int32_t plan_kernels = 0, plan_fused = 0, plan_wrap = 0;
+  int32_t plan_kernels = 0, plan_fused = 0, plan_wrap = 0, plan_host_streamed = 0;
   int64_t plan_streams = 0, plan_blocks_per_sm = 0;
   // phase profiling (bpbc_sw_profile): 4 events per recorded call
   bool profiling = false;
@@ -146,7 +157,7 @@ struct Plan {
   int ops;
 };
 
-int make_plan(int mq, int c1, int c2, int g, int S, bool no_exact_run, Plan* p) {
+int make_plan(int mq, int c1, int c2, int g, int S, bool no_exact_run, bool force_width, Plan* p) {
   if (mq <= 32) p->rl = 0;
   else if (mq <= 64) p->rl = 1;
   else if (mq <= 128) p->rl = 2;
@@ -164,7 +175,7 @@ int make_plan(int mq, int c1, int c2, int g, int S, bool no_exact_run, Plan* p) 
   int s_sat = bit_length(int64_t(c1) * mq);
   if (s_sat < bit_length(cmax)) s_sat = bit_length(cmax);
   if (s_sat < BPBC_MIN_SCORE_BITS) s_sat = BPBC_MIN_SCORE_BITS;
-  if (s_sat > S) s_sat = S;
+  if (s_sat > S || force_width) s_sat = S;  // (force_width: circuit-depth studies, DESIGN 6)
   const int cost_sat = 11 * s_sat + 2;
   if (g >= c2) {
     // exact offset circuit at the width no value can exceed: compile-time
@@ -172,6 +183,7 @@ int make_plan(int mq, int c1, int c2, int g, int S, bool no_exact_run, Plan* p) 
     // than the saturating circuit
     int s_ex = bit_length(int64_t(c1) * mq + g);
     if (s_ex < BPBC_MIN_SCORE_BITS) s_ex = BPBC_MIN_SCORE_BITS;
+    if (force_width && S > s_ex) s_ex = S;  // still exact at any width above
     const int cost_ex = spec ? 10 * s_ex : 12 * s_ex + 1;
     const int cost_sat_k = spec ? cost_sat : 13 * s_sat + 4;
     if (s_ex <= BPBC_MAX_SCORE_BITS && cost_ex <= cost_sat_k && (spec || !no_exact_run)) {
@@ -351,7 +363,7 @@ void split_streams(const bpbc_sw_ctx* ctx, int nt, int64_t nb, int64_t nbw, Disp
 
 int make_dispatch(bpbc_sw_ctx* ctx, int64_t P, int mq, int nt, int c1, int c2, int g, int S,
                   int mode, Dispatch* d) {
-  int rc = make_plan(mq, c1, c2, g, S, ctx->opt_no_exact_run, &d->plan);
+  int rc = make_plan(mq, c1, c2, g, S, ctx->opt_no_exact_run, ctx->opt_force_width, &d->plan);
   if (rc != BPBC_OK) return rc;
   std::call_once(g_table_once, init_table);
   const Plan& plan = d->plan;
@@ -568,6 +580,7 @@ struct RunOut {
   uint32_t* mask = nullptr;      //   [ceil(P/32)] flag words
   int64_t* indices = nullptr;    //   optional ascending flagged pair indices
   int64_t* count = nullptr;      //   optional number of flagged pairs
+  const uint32_t* progress = nullptr;  // host-streamed inputs (fused kernel): waves ready
 };
 
 // Enqueue pack -> sweep -> extract (or the filter epilogue) on device buffers
@@ -636,6 +649,7 @@ int run_device(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, const u
   a.span = dsp.span;
   a.snap = reinterpret_cast<uint32_t*>(ws + lay.snap_off);
   a.snap_flag = reinterpret_cast<uint32_t*>(ws + lay.sflag_off);
+  a.progress = o.progress;
   KRun kr;
   memset(&kr, 0, sizeof(kr));
   const int Wd = plan.width;
@@ -757,6 +771,109 @@ int slot_events(bpbc_sw_ctx* ctx, HostSlot& s) {
   return BPBC_OK;
 }
 
+// cuStreamWriteValue32 (driver API, through the runtime's entry-point query:
+// no link against libcuda): a 32-bit store ordered after the stream's
+// previous work, with a memory barrier (flags 0), done by the GPU front end.
+typedef int (*WriteValue32Fn)(void* stream, unsigned long long addr, unsigned int value,
+                              unsigned int flags);
+WriteValue32Fn write_value32() {
+  static WriteValue32Fn fn = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      f = nullptr;
+    cudaGetLastError();
+    return reinterpret_cast<WriteValue32Fn>(f);
+  }();
+  return fn;
+}
+
+// Host path as ONE streamed launch (fused group-granular plans): the whole
+// batch's device buffers are filled wave by wave on the copy-in stream (a
+// wave = the h-th group of every sweep stream = S consecutive groups, since
+// the fused kernel assigns groups to streams strided), each followed by a
+// device-side write of the wave count to `progress`; the sweep runs
+// concurrently on the compute stream and polls `progress` before it touches
+// a wave (SweepArgs::progress).  No per-chunk pipeline fill, the copy
+// overlaps the kernels from the first wave on, and only the first wave's
+// copy is exposed.  Returns BPBC_ERR_UNSUPPORTED when the device cannot do
+// stream memory writes (the caller then uses the chunked path).
+int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, const uint8_t* ty,
+                  int64_t P, int mq, int nt, int c1, int c2, int g, int64_t qs, int64_t ts,
+                  int32_t* out_scores, bool packed2) {
+  WriteValue32Fn wv = write_value32();
+  if (!wv) return BPBC_ERR_UNSUPPORTED;
+  cudaError_t e;
+  int rc;
+  cudaStream_t cin = ctx->hs_in, comp = ctx->hs_comp;
+  const size_t need = size_t(layout(P, mq, nt, &dsp, false).total);
+  if ((rc = grow_async(ctx, (void**)&ctx->s_q, &ctx->s_q_bytes, size_t(P * qs), comp,
+                       "cudaMallocAsync(q)")) != BPBC_OK ||
+      (rc = grow_async(ctx, (void**)&ctx->s_t, &ctx->s_t_bytes, size_t(P * ts), comp,
+                       "cudaMallocAsync(t)")) != BPBC_OK ||
+      (rc = grow_async(ctx, (void**)&ctx->s_out, &ctx->s_out_bytes, size_t(P) * 4, comp,
+                       "cudaMallocAsync(out)")) != BPBC_OK ||
+      (rc = grow_async(ctx, &ctx->s_ws, &ctx->s_ws_bytes, need, comp,
+                       "cudaMallocAsync(workspace)")) != BPBC_OK)
+    return rc;
+  cudaEvent_t* evs[3] = {&ctx->ev_reset, &ctx->ev_c0, &ctx->ev_c1};
+  for (int i = 0; i < 3; ++i)
+    if (!*evs[i] && (e = (i == 0 ? cudaEventCreateWithFlags(evs[i], cudaEventDisableTiming)
+                                 : cudaEventCreate(evs[i]))) != cudaSuccess)
+      return cuda_fail(ctx, e, "event");
+  if (!ctx->progress && (e = cudaMalloc(&ctx->progress, 256)) != cudaSuccess)
+    return cuda_fail(ctx, e, "cudaMalloc(progress)");
+  // progress = 0 before the kernel starts; the copy stream's first write
+  // comes after the reset (and after the allocations above)
+  if ((e = cudaMemsetAsync(ctx->progress, 0, 4, comp)) != cudaSuccess ||
+      (e = cudaEventRecord(ctx->ev_reset, comp)) != cudaSuccess ||
+      (e = cudaStreamWaitEvent(cin, ctx->ev_reset, 0)) != cudaSuccess)
+    return cuda_fail(ctx, e, "progress reset");
+  // copy-in: waves, growing 1, 1, 2, 4, ... (the first wave's copy is the
+  // only exposed one; later writes cover several waves)
+  const int64_t S = dsp.streams;
+  const int64_t G = (P + 31) / 32;
+  const int64_t waves = (G + S - 1) / S;
+  cudaEventRecord(ctx->ev_c0, cin);
+  int64_t w0 = 0, step = 1;
+  while (w0 < waves) {
+    const int64_t w1 = w0 + step < waves ? w0 + step : waves;
+    const int64_t p0 = w0 * S * 32, p1 = w1 * S * 32 < P ? w1 * S * 32 : P;
+    e = cudaMemcpyAsync(ctx->s_q + p0 * qs, qx + p0 * qs, size_t((p1 - p0) * qs),
+                        cudaMemcpyHostToDevice, cin);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(ctx->s_t + p0 * ts, ty + p0 * ts, size_t((p1 - p0) * ts),
+                          cudaMemcpyHostToDevice, cin);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "H2D");
+    if (wv(cin, reinterpret_cast<unsigned long long>(ctx->progress), unsigned(w1), 0) != 0) {
+      cudaGetLastError();
+      return BPBC_ERR_UNSUPPORTED;
+    }
+    w0 = w1;
+    step = w0 < 2 ? 1 : (step * 2 < 8 ? step * 2 : 8);
+  }
+  cudaEventRecord(ctx->ev_c1, cin);
+  RunOut o;
+  o.scores = ctx->s_out;
+  o.progress = ctx->progress;
+  rc = run_device(ctx, dsp, ctx->s_q, ctx->s_t, P, mq, nt, c1, c2, g, o,
+                  static_cast<uint8_t*>(ctx->s_ws), comp, packed2);
+  if (rc != BPBC_OK) return rc;
+  if ((e = cudaMemcpyAsync(out_scores, ctx->s_out, size_t(P) * 4, cudaMemcpyDeviceToHost, comp)) !=
+      cudaSuccess)
+    return cuda_fail(ctx, e, "D2H");
+  if ((e = cudaStreamSynchronize(comp)) != cudaSuccess ||
+      (e = cudaStreamSynchronize(cin)) != cudaSuccess)
+    return cuda_fail(ctx, e, "sync");
+  float ms = 0;
+  if (cudaEventElapsedTime(&ms, ctx->ev_c0, ctx->ev_c1) == cudaSuccess && ms > 0 &&
+      P * (qs + ts) > (1 << 20))
+    ctx->h2d_bps = double(P * (qs + ts)) / (ms * 1e-3);
+  cudaGetLastError();
+  return BPBC_OK;
+}
+
 int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t* target,
                           int64_t num_pairs, int32_t m, int32_t n, int32_t match,
                           int32_t mismatch, int32_t gap, int32_t score_bits, int32_t* out_scores,
@@ -788,6 +905,35 @@ int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t*
   if ((rc = make_dispatch(ctx, num_pairs, mq, nt, c1, c2, g, score_bits, kModeMax, &full)) !=
       BPBC_OK)
     return rc;
+  // fused group-granular plans: one streamed launch (host_streamed)
+  if (full.fused && !full.wrap && full.mw < 0 && !ctx->opt_chunked_host) {
+    // results: straight into a pinned output, else through pinned staging
+    cudaPointerAttributes pa;
+    const bool pinned = cudaPointerGetAttributes(&pa, out_scores) == cudaSuccess &&
+                        pa.type == cudaMemoryTypeHost;
+    cudaGetLastError();
+    int32_t* dst = out_scores;
+    if (!pinned) {
+      const size_t ob = size_t(num_pairs) * 4;
+      if (ctx->h_out_bytes < ob) {
+        if (ctx->h_out) cudaFreeHost(ctx->h_out);
+        ctx->h_out = nullptr;
+        ctx->h_out_bytes = 0;
+        if ((e = cudaMallocHost(&ctx->h_out, ob)) != cudaSuccess)
+          return cuda_fail(ctx, e, "cudaMallocHost(out staging)");
+        ctx->h_out_bytes = ob;
+      }
+      dst = ctx->h_out;
+    }
+    rc = host_streamed(ctx, full, qx, ty, num_pairs, mq, nt, c1, c2, g, qs, ts, dst, packed2);
+    if (rc == BPBC_OK) {
+      if (!pinned) memcpy(out_scores, ctx->h_out, size_t(num_pairs) * 4);
+      ctx->plan_host_streamed = 1;
+      return BPBC_OK;
+    }
+    if (rc != BPBC_ERR_UNSUPPORTED) return rc;
+  }
+  ctx->plan_host_streamed = 0;
   // (few groups: a chunk of them would leave SMSPs idle -- no chunking)
   const int64_t wave_pairs = full.wrap ? num_pairs : full.streams * 32;
   // Chunk plan from the measured rates.  Every chunk's
@@ -982,6 +1128,8 @@ int bpbc_sw_init(int cuda_device, bpbc_sw_ctx** out_ctx) {
   ctx->opt_max_blocks = env_int("BPBC_MAX_BLOCKS_PER_SM", 0);
   ctx->opt_no_exact_run = env_int("BPBC_NO_EXACT_RUN", 0) != 0;
   ctx->opt_wrap = env_int("BPBC_WRAP", -1);
+  ctx->opt_chunked_host = env_int("BPBC_CHUNKED_HOST", 0) != 0;
+  ctx->opt_force_width = env_int("BPBC_FORCE_WIDTH", 0) != 0;
   DeviceGuard dg(cuda_device);
   e = cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
   if (e == cudaSuccess) e = cudaMalloc(&ctx->d_flags, sizeof(uint32_t));
@@ -1015,6 +1163,14 @@ int bpbc_sw_destroy(bpbc_sw_ctx* ctx) {
     if (s) cudaStreamSynchronize(s);
   if (ctx->buf_used) cudaEventSynchronize(ctx->buf_ev);
   if (ctx->ws) cudaFreeAsync(ctx->ws, ctx->aux);
+  {
+    void* bufs[4] = {ctx->s_q, ctx->s_t, ctx->s_out, ctx->s_ws};
+    for (void* p : bufs)
+      if (p) cudaFreeAsync(p, ctx->aux);
+    cudaEvent_t evs[3] = {ctx->ev_reset, ctx->ev_c0, ctx->ev_c1};
+    for (cudaEvent_t ev : evs)
+      if (ev) cudaEventDestroy(ev);
+  }
   for (auto& s : ctx->slots) {
     void* bufs[4] = {s.dq, s.dt, s.dout, s.ws};
     for (void* p : bufs)
@@ -1027,6 +1183,7 @@ int bpbc_sw_destroy(bpbc_sw_ctx* ctx) {
   for (cudaStream_t s : {ctx->hs_in, ctx->hs_comp, ctx->hs_out})
     if (s) cudaStreamDestroy(s);
   if (ctx->d_flags) cudaFree(ctx->d_flags);
+  if (ctx->progress) cudaFree(ctx->progress);
   if (ctx->h_flags) cudaFreeHost(ctx->h_flags);
   if (ctx->h_out) cudaFreeHost(ctx->h_out);
   if (ctx->aux) cudaStreamDestroy(ctx->aux);
@@ -1241,10 +1398,12 @@ int bpbc_sw_last_launches(bpbc_sw_ctx* ctx, int32_t* kernels, int32_t* fused) {
   return BPBC_OK;
 }
 
-int bpbc_sw_last_schedule(bpbc_sw_ctx* ctx, int32_t* wrap, int64_t* blocks_per_sm) {
+int bpbc_sw_last_schedule(bpbc_sw_ctx* ctx, int32_t* wrap, int64_t* blocks_per_sm,
+                          int32_t* host_streamed) {
   if (!ctx) return BPBC_ERR_INVALID_ARG;
   if (wrap) *wrap = ctx->plan_wrap;
   if (blocks_per_sm) *blocks_per_sm = ctx->plan_blocks_per_sm;
+  if (host_streamed) *host_streamed = ctx->plan_host_streamed;
   return BPBC_OK;
 }
 

@@ -39,7 +39,9 @@ struct SweepArgs {
   int m, n;          // query rows (m <= L*R), target columns
   int64_t streams;   // number of group streams (one per L lanes)
   int64_t base;      // groups per stream: base or base+1
-  int64_t rem;       //   (the first rem streams get base+1)
+  int64_t rem;       //   (the first rem streams get base+1; planes / multi-warp /
+                     //   striped kernels: contiguous ranges; the fused kernel:
+                     //   stream st takes groups st, st + streams, ...)
   int64_t steps;     // wavefront steps = (base + (rem>0)) * stripes * n + L
   // long-query (striped) kernel only
   // fused single-warp kernel: the caller's raw codes (query rows m, target
@@ -66,6 +68,10 @@ struct SweepArgs {
   int64_t span;         // columns per stream (multiple of 32, >= n)
   uint32_t* snap;       // [streams][kSnapWords][32] warp-state snapshots
   uint32_t* snap_flag;  // [streams] 1 once snapshot k is written (zeroed per call)
+  // Host-streamed inputs (fused group-granular kernel, bpbc_sw_score_batch_host):
+  // wave h (the h-th group of every stream: groups [h streams, (h+1) streams))
+  // is in device memory once *progress > h; nullptr = inputs resident.
+  const uint32_t* progress;
 };
 
 // Words of one lane's warp-state snapshot (wrap-around schedule): R rows x S

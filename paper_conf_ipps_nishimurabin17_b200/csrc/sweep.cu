@@ -92,14 +92,15 @@ __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wai
 
 // Target chunk that straddles two groups of a stream (only when n % 32 != 0):
 // lane k gathers positions col.. of pair 32g+k, continuing into pair
-// 32(g+1)+k after the row end; folded H / L as tr_load_fold.  Out of line:
-// one copy per object instead of one per kernel instantiation.
+// 32 g_next + k (the stream's next group) after the row end; folded H / L as
+// tr_load_fold.  Out of line: one copy per object instead of one per kernel
+// instantiation.
 __device__ __noinline__ uint3 gather_straddle(const uint8_t* traw, int64_t tstride, int n,
-                                              int64_t P, int64_t g, bool has_next, int col,
-                                              int lane, bool packed2) {
+                                              int64_t P, int64_t g, int64_t g_next, bool has_next,
+                                              int col, int lane, bool packed2) {
   uint32_t H, L, bad = 0;
   uint32_t w[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-  const int64_t row0 = g * 32 + lane, row1 = (g + 1) * 32 + lane;
+  const int64_t row0 = g * 32 + lane, row1 = g_next * 32 + lane;
 #pragma unroll
   for (int i = 0; i < 32; ++i) {
     const bool next = col + i >= n;  // past this group's last column
@@ -119,6 +120,16 @@ __device__ __noinline__ uint3 gather_straddle(const uint8_t* traw, int64_t tstri
   if (packed2) tr_fold_packed2(w[0], w[1], H, L);
   else tr_fold_u8(w, H, L, bad);
   return make_uint3(H, L, bad);  // by value: registers, no stack frame at the call
+}
+
+// Acquire / release accesses of the progress and snapshot flags.
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
 // ---------------------------------------------------------------------------
@@ -141,6 +152,7 @@ struct FusedLane {
   int gi;             // my current group within the (sub-)stream
   int gsn;            // group ends stored in this (sub-)stream
   uint32_t* mdst;     // my partial-max slot of the current group, advanced at every switch
+  int mstep;          // words from one group's slot to the next group's (kMW x group stride)
   const uint2* xrow;  // my query-plane slot 0 in the shared ring (+ slot * 32 * R)
 
   __device__ __forceinline__ void reset(int sl) {
@@ -184,7 +196,7 @@ struct FusedLane {
 #pragma unroll
         for (int i = 0; i < S; ++i) st_if(mdst + i, M[i], st);
       }
-      mdst += st * kMW;
+      mdst += st * mstep;
       gi += sw ? 1 : 0;
       flag = mul_lo(flag, keep);
 #pragma unroll
@@ -208,7 +220,7 @@ struct FusedLane {
 #pragma unroll
           for (int i = 0; i < S; ++i) mdst[i] = M[i];
         }
-        mdst += kMW;
+        mdst += mstep;
       }
       ++gi;
       flag = mul_lo(flag, z0);
@@ -332,14 +344,33 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   const int64_t warp = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   if (warp * SEGS >= a.streams) return;  // uniform per warp
 
-  // groups of segment s's stream (uniform per warp for each s)
+  // groups of segment s's stream (uniform per warp for each s): stream st
+  // takes the groups st, st + streams, st + 2 streams, ... (strided, so the
+  // h-th groups of all streams -- one "wave" -- are contiguous: the
+  // host-streamed path copies the input wave by wave, a.progress)
+  const int64_t gstr = a.streams;
   auto seg_range = [&](int s, int64_t& gbs, int64_t& gss) {
     const int64_t st = warp * SEGS + s;
     gss = 0;
     gbs = 0;
     if (st < a.streams) {
-      gss = a.base + (st < a.rem ? 1 : 0);
-      gbs = st * a.base + (st < a.rem ? st : a.rem);
+      gss = (a.G - st + gstr - 1) / gstr;
+      gbs = st;
+    }
+  };
+  // host-streamed inputs: wave h (group index h of every stream) may be read
+  // once the copy stream has published a.progress > h (warp-uniform poll)
+  uint32_t ready = a.progress ? 0u : 0xFFFFFFFFu;
+  auto wait_wave = [&](int64_t h) {
+    if (uint64_t(h) >= ready) {
+      while (true) {
+        const uint32_t v = ld_acquire_gpu(a.progress);
+        if (!__any_sync(0xFFFFFFFFu, uint64_t(v) <= uint64_t(h))) {
+          ready = v;
+          break;
+        }
+        __nanosleep(512);
+      }
     }
   };
   int64_t Gs, gb;
@@ -370,12 +401,14 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     if (v0 >= 0 && v0 < gss * a.n) {
       const int64_t h = v0 / a.n;
       const int col = int(v0 - h * a.n);
-      const int64_t g = gbs + h;
+      const int64_t g = gbs + h * gstr;
       if (col + 32 <= a.n) {
+        wait_wave(h);
         tr_load_fold(a.traw, a.tstride, a.n, g * 32 + lane, a.P, col, packed2, Hw, Lw, bad);
       } else {  // the chunk straddles two groups (n % 32 != 0; n >= 48)
-        const uint3 r3 = gather_straddle(a.traw, a.tstride, a.n, a.P, g, h + 1 < gss, col, lane,
-                                         packed2);
+        wait_wave(h + 1 < gss ? h + 1 : h);
+        const uint3 r3 = gather_straddle(a.traw, a.tstride, a.n, a.P, g, g + gstr, h + 1 < gss,
+                                         col, lane, packed2);
         Hw = r3.x;
         Lw = r3.y;
         bad |= r3.z;
@@ -390,8 +423,9 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   auto build_x = [&](int s, int64_t h) {
     int64_t gbs, gss;
     seg_range(s, gbs, gss);
-    int64_t g = gbs + h;
-    g = g < a.G ? g : a.G - 1;
+    int64_t g = gbs + h * gstr;
+    if (g >= a.G) g = gbs < a.G ? gbs : a.G - 1;  // past the stream's last group: unused
+    else wait_wave(h);
 #pragma unroll
     for (int c = 0; c < XCH; ++c) {
       uint32_t Hw = 0, Lw = 0;
@@ -404,6 +438,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
 
   ln.gsn = int(Gs);  // groups of my stream (< 2^31: P < 2^36)
   ln.mdst = a.Mpart + (gb * L + sl) * (ln.kMW / L);
+  ln.mstep = int(ln.kMW * gstr);
   ln.xrow = &xr[0][lane][0];
 
   // prologue: the first group's query planes, target chunks -1 (zeros), 0, 1
@@ -460,14 +495,6 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
 // makes the tail start at least (span - n) columns after the head ends.
 // Per sub-stream the body is sw_sweep_kernel's (same transposes, rings,
 // switch handling and circuits).
-__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
-  uint32_t v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
 
 
 // (no occupancy floor: the schedule runs it with few blocks per SM; the
@@ -571,6 +598,7 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
     ln.reset(lane);
     ln.gsn = gs;
     ln.mdst = a.Mpart + (g0 * L + lane) * (ln.kMW / L);
+    ln.mstep = ln.kMW;
 
     // ---- prologue: first group's query planes, target chunks -1 (zeros, or
     // the columns before c0 when resuming), 0, 1

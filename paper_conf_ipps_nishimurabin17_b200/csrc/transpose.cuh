@@ -75,33 +75,13 @@ __device__ __forceinline__ void tr_butterfly(uint32_t& H, uint32_t& L, int lane)
   }
 }
 
-// The (pre-butterfly) H / L words of positions [c0, c0 + 32) of one row of a
-// raw input (u8 codes or 2-bit packed, `stride` bytes per row, `len`
-// positions): zeros past the row end and for rows >= nrows.  16-byte loads
-// when the row segment is aligned and whole.
-__device__ __forceinline__ void tr_load_fold(const uint8_t* base, int64_t stride, int len,
-                                             int64_t row, int64_t nrows, int c0, bool packed2,
-                                             uint32_t& H, uint32_t& L, uint32_t& bad) {
-  if (packed2) {
-    uint32_t w[2] = {0u, 0u};
-    if (row < nrows) {
-      const uint8_t* p = base + row * stride + c0 / 4;
-      if (c0 + 32 <= len && ((reinterpret_cast<uintptr_t>(p) & 7) == 0)) {
-        const uint2 v = *reinterpret_cast<const uint2*>(p);
-        w[0] = v.x;
-        w[1] = v.y;
-      } else {
-#pragma unroll
-        for (int q = 0; q < 2; ++q)
-#pragma unroll
-          for (int bb = 0; bb < 4; ++bb)
-            if (c0 + 16 * q + 4 * bb < len) w[q] |= uint32_t(p[4 * q + bb]) << (8 * bb);
-      }
-    }
-    tr_fold_packed2(w[0], w[1], H, L);
-    return;
-  }
-  uint32_t w[8];
+// Raw words of positions [c0, c0 + 32) of one row of a raw input (`stride`
+// bytes per row, `len` positions): zeros past the row end and for rows >=
+// nrows.  u8 codes: 8 words (byte b of w[q] = position 4q + b), two 16-byte
+// streaming loads when the row segment is 16-byte aligned and whole; 2-bit
+// packed: 2 words (positions 0..15, 16..31), one 8-byte load when aligned.
+__device__ __forceinline__ void tr_load_u8(const uint8_t* base, int64_t stride, int len,
+                                           int64_t row, int64_t nrows, int c0, uint32_t (&w)[8]) {
 #pragma unroll
   for (int q = 0; q < 8; ++q) w[q] = 0u;
   if (row < nrows) {
@@ -119,6 +99,39 @@ __device__ __forceinline__ void tr_load_fold(const uint8_t* base, int64_t stride
           if (c0 + 4 * q + bb < len) w[q] |= uint32_t(p[4 * q + bb]) << (8 * bb);
     }
   }
+}
+__device__ __forceinline__ void tr_load_p2(const uint8_t* base, int64_t stride, int len,
+                                           int64_t row, int64_t nrows, int c0, uint32_t (&w)[2]) {
+  w[0] = w[1] = 0u;
+  if (row < nrows) {
+    const uint8_t* p = base + row * stride + c0 / 4;
+    if (c0 + 32 <= len && ((reinterpret_cast<uintptr_t>(p) & 7) == 0)) {
+      const uint2 v = *reinterpret_cast<const uint2*>(p);
+      w[0] = v.x;
+      w[1] = v.y;
+    } else {
+#pragma unroll
+      for (int q = 0; q < 2; ++q)
+#pragma unroll
+        for (int bb = 0; bb < 4; ++bb)
+          if (c0 + 16 * q + 4 * bb < len) w[q] |= uint32_t(p[4 * q + bb]) << (8 * bb);
+    }
+  }
+}
+
+// The (pre-butterfly) H / L words of positions [c0, c0 + 32) of one row of a
+// raw input (u8 codes or 2-bit packed).
+__device__ __forceinline__ void tr_load_fold(const uint8_t* base, int64_t stride, int len,
+                                             int64_t row, int64_t nrows, int c0, bool packed2,
+                                             uint32_t& H, uint32_t& L, uint32_t& bad) {
+  if (packed2) {
+    uint32_t w[2];
+    tr_load_p2(base, stride, len, row, nrows, c0, w);
+    tr_fold_packed2(w[0], w[1], H, L);
+    return;
+  }
+  uint32_t w[8];
+  tr_load_u8(base, stride, len, row, nrows, c0, w);
   tr_fold_u8(w, H, L, bad);
 }
 

@@ -13,6 +13,7 @@ oracle; exits non-zero on a mismatch.
 """
 import os
 import sys
+import threading
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))  # repo root
 sys.path.insert(0, ROOT)
@@ -72,6 +73,47 @@ def main():
     got = bpbc.score_batch_wordwise(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV)).cpu()
     bad += check("wordwise", got.numpy(), oracle.sw_batch(q, t, 2, -1, -1))
     bad += check("host path", bpbc.score_batch_host(q, t, 2, -1, -1, 9), want)
+    # wrap-around schedule (snapshot hand-off through global memory with
+    # acquire/release flags), forced on a 600-group batch in a thread whose
+    # ctx reads BPBC_WRAP=1 / one block per SM at init
+    q, t = synth.gen_pairs(79, 600 * 32, 128, 256, planted=True)
+    res = {}
+
+    def wrap_case():
+        res["got"] = bpbc.score_batch(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV),
+                                      score_bits=9).cpu().numpy()
+        res["plan"] = bpbc.last_plan(0)
+        bpbc.release_thread_ctx(0)
+
+    os.environ.update({"BPBC_WRAP": "1", "BPBC_MAX_BLOCKS_PER_SM": "1"})
+    th = threading.Thread(target=wrap_case)
+    th.start()
+    th.join()
+    for k in ("BPBC_WRAP", "BPBC_MAX_BLOCKS_PER_SM"):
+        os.environ.pop(k, None)
+    bad += check(f"wrap-around plan={res.get('plan')}", res.get("got"),
+                 oracle.sw_batch(q, t, 2, -1, -1, score_bits=9))
+    # two streams through one ctx with the ctx-owned workspace (workspace =
+    # NULL): the second call waits for the first one's use of it
+    qa, ta = synth.gen_pairs(80, 300, 64, 64, planted=True)
+    qb, tb = synth.gen_pairs(81, 500, 64, 96, planted=True)
+    s1, s2 = torch.cuda.Stream(DEV), torch.cuda.Stream(DEV)
+    da = [torch.from_numpy(x).to(DEV) for x in (qa, ta)]
+    db = [torch.from_numpy(x).to(DEV) for x in (qb, tb)]
+    torch.cuda.synchronize()
+    with torch.cuda.stream(s1):
+        oa = bpbc.score_batch(*da, score_bits=8, stream=s1)
+    with torch.cuda.stream(s2):
+        ob = bpbc.score_batch(*db, score_bits=8, stream=s2)
+    torch.cuda.synchronize()
+    bad += check("two streams, ctx workspace (a)", oa.cpu().numpy(),
+                 oracle.sw_batch(qa, ta, 2, -1, -1, score_bits=8))
+    bad += check("two streams, ctx workspace (b)", ob.cpu().numpy(),
+                 oracle.sw_batch(qb, tb, 2, -1, -1, score_bits=8))
+    # the standalone transpose kernel (W2B) against its definition
+    codes = np.random.default_rng(5).integers(0, 4, size=(70, 300), dtype=np.uint8)
+    planes = bpbc.pack(torch.from_numpy(codes).to(DEV)).cpu().numpy().view(np.uint32)
+    bad += check("pack", planes, oracle.pack_planes(codes))
     torch.cuda.synchronize()
     print("sanitize_run:", "PASS" if bad == 0 else "FAIL", flush=True)
     sys.exit(1 if bad else 0)

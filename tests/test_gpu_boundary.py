@@ -169,3 +169,80 @@ def test_multi_device_driver_releases_ctxs_and_returns_flags():
     assert len(api._ctxs) == before  # worker ctxs were destroyed with their threads
     assert flags[1] & _lib.BPBC_FLAG_BAD_BASE and not flags[0]
     np.testing.assert_array_equal(got, oracle.sw_batch(q, t2 & 3, 2, -1, -1, score_bits=8))
+
+
+@pytest.mark.parametrize("P,m,n,packed2", [(300000, 128, 128, False), (300000, 128, 128, True),
+                                           (200001, 64, 100, False), (90000, 40, 1000, True),
+                                           (150000, 200, 256, False)])
+def test_host_streamed_launch(P, m, n, packed2):
+    """bpbc_sw_score_batch_host as one streamed launch (waves copied on the
+    copy stream, progress writes, the sweep polling them): equal to the
+    device path; ragged P, n % 32 != 0 (chunks straddling a stream's
+    consecutive -- strided -- groups), L = 16 and R = 8 tilings."""
+    q, t = synth.gen_pairs(9500 + m + n, P, m, n, planted=True)
+    s = bpbc.default_score_bits(2, m, n)
+    if packed2:
+        got = bpbc.score_batch_host_packed2(synth.pack2bit(q), synth.pack2bit(t), m, n, 2, -1, -1, s)
+    else:
+        got = bpbc.score_batch_host(q, t, 2, -1, -1, s)
+    assert bpbc.last_plan(0)["host_streamed"]
+    dev = bpbc.score_batch(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV),
+                           score_bits=s).cpu().numpy()
+    np.testing.assert_array_equal(got, dev)
+    idx = np.arange(0, P, 53)
+    np.testing.assert_array_equal(got[idx], oracle.sw_batch(q[idx], t[idx], 2, -1, -1, score_bits=s))
+
+
+def test_host_chunked_knob_matches_streamed():
+    """BPBC_CHUNKED_HOST=1 (a ctx made in a thread with it set) takes the
+    chunked path; both give the oracle's scores."""
+    import os
+    import threading
+    P, m, n = 120000, 96, 128
+    q, t = synth.gen_pairs(9600, P, m, n, planted=True)
+    box = {}
+
+    def run():
+        box["got"] = bpbc.score_batch_host(q, t, 2, -1, -1, 9)
+        box["plan"] = bpbc.last_plan(0)
+        bpbc.release_thread_ctx(0)
+
+    os.environ["BPBC_CHUNKED_HOST"] = "1"
+    try:
+        th = threading.Thread(target=run)
+        th.start()
+        th.join()
+    finally:
+        os.environ.pop("BPBC_CHUNKED_HOST", None)
+    assert not box["plan"]["host_streamed"]
+    streamed = bpbc.score_batch_host(q, t, 2, -1, -1, 9)
+    np.testing.assert_array_equal(box["got"], streamed)
+    idx = np.arange(0, P, 41)
+    np.testing.assert_array_equal(streamed[idx], oracle.sw_batch(q[idx], t[idx], 2, -1, -1,
+                                                                 score_bits=9))
+
+
+@pytest.mark.parametrize("s", [10, 12, 16])
+def test_force_width_knob(s):
+    """BPBC_FORCE_WIDTH=1 evaluates the circuit at score_bits (above s_exact
+    the exact circuit is still exact): same scores, plan width = s."""
+    import os
+    import threading
+    q, t = synth.gen_pairs(9700 + s, 5000, 64, 64, planted=True)
+    box = {}
+
+    def run():
+        box["got"] = bpbc.score_batch(torch.from_numpy(q).to(DEV), torch.from_numpy(t).to(DEV),
+                                      score_bits=s).cpu().numpy()
+        box["plan"] = bpbc.last_plan(0)
+        bpbc.release_thread_ctx(0)
+
+    os.environ["BPBC_FORCE_WIDTH"] = "1"
+    try:
+        th = threading.Thread(target=run)
+        th.start()
+        th.join()
+    finally:
+        os.environ.pop("BPBC_FORCE_WIDTH", None)
+    assert box["plan"]["width"] == s
+    np.testing.assert_array_equal(box["got"], oracle.sw_batch(q, t, 2, -1, -1, score_bits=s))

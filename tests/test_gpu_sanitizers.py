@@ -1,0 +1,31 @@
+"""compute-sanitizer over every kernel family: memcheck,
+racecheck, synccheck and initcheck run tests/sanitize_run.py (small cases of
+every kernel family, each checked against the oracle) and must report no
+error.  BPBC_SKIP_SANITIZERS=1 skips them (they take minutes)."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+pytestmark = [pytest.mark.gpu,
+              pytest.mark.skipif(shutil.which("compute-sanitizer") is None,
+                                 reason="no compute-sanitizer"),
+              pytest.mark.skipif(os.environ.get("BPBC_SKIP_SANITIZERS") == "1",
+                                 reason="BPBC_SKIP_SANITIZERS=1")]
+
+CLEAN = {"memcheck": "ERROR SUMMARY: 0 errors", "racecheck": "0 hazards displayed",
+         "synccheck": "ERROR SUMMARY: 0 errors", "initcheck": "ERROR SUMMARY: 0 errors"}
+
+
+@pytest.mark.parametrize("tool", sorted(CLEAN))
+def test_sanitizer_clean(tool):
+    r = subprocess.run(["compute-sanitizer", "--tool", tool, sys.executable,
+                        os.path.join(ROOT, "tests", "sanitize_run.py")],
+                       capture_output=True, text=True, timeout=1500, cwd=ROOT)
+    out = r.stdout + r.stderr
+    assert "sanitize_run: PASS" in out, out[-3000:]
+    assert CLEAN[tool] in out, out[-3000:]
+    assert r.returncode == 0, out[-3000:]

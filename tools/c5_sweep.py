@@ -82,7 +82,7 @@ def main():
             gcups = P * m * n * args.steps / (t_ms / 1e3) / 1e9
             sweep_ms = ph["swa_ms"] / max(1, ph["calls"])
             word_cells = (P + 31) // 32 * m * n
-            peak = bench.peak_alu_tops(clocks.get("sm_max_mhz") or 1965.0)
+            peak = bench.measured_lop3_peak()[0]
             frac = plan["ops_per_word_cell"] * word_cells / (sweep_ms / 1e3) / 1e12 / peak
             got = out.cpu().numpy()
             cap = (1 << s) - 1
