@@ -580,7 +580,8 @@ struct RunOut {
   uint32_t* mask = nullptr;      //   [ceil(P/32)] flag words
   int64_t* indices = nullptr;    //   optional ascending flagged pair indices
   int64_t* count = nullptr;      //   optional number of flagged pairs
-  const uint32_t* progress = nullptr;  // host-streamed inputs (fused kernel): waves ready
+  const uint32_t* progress = nullptr;  // host-streamed inputs: waves ready (SweepArgs)
+  int64_t blk_first = 0, blk_rest = 0;  //   wrap-around copy timeline blocks
 };
 
 // Enqueue pack -> sweep -> extract (or the filter epilogue) on device buffers
@@ -650,6 +651,8 @@ int run_device(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, const u
   a.snap = reinterpret_cast<uint32_t*>(ws + lay.snap_off);
   a.snap_flag = reinterpret_cast<uint32_t*>(ws + lay.sflag_off);
   a.progress = o.progress;
+  a.blk_first = o.blk_first;
+  a.blk_rest = o.blk_rest;
   KRun kr;
   memset(&kr, 0, sizeof(kr));
   const int Wd = plan.width;
@@ -830,36 +833,110 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
       (e = cudaEventRecord(ctx->ev_reset, comp)) != cudaSuccess ||
       (e = cudaStreamWaitEvent(cin, ctx->ev_reset, 0)) != cudaSuccess)
     return cuda_fail(ctx, e, "progress reset");
-  // copy-in: waves, growing 1, 1, 2, 4, ... (the first wave's copy is the
-  // only exposed one; later writes cover several waves)
+  // The copy-in plan, as waves, each closed by a progress write of the waves
+  // done; wave 0 is enqueued before the kernel, the rest after it (their
+  // API calls then overlap the kernel).
   const int64_t S = dsp.streams;
   const int64_t G = (P + 31) / 32;
-  const int64_t waves = (G + S - 1) / S;
-  cudaEventRecord(ctx->ev_c0, cin);
-  int64_t w0 = 0, step = 1;
-  while (w0 < waves) {
-    const int64_t w1 = w0 + step < waves ? w0 + step : waves;
-    const int64_t p0 = w0 * S * 32, p1 = w1 * S * 32 < P ? w1 * S * 32 : P;
-    e = cudaMemcpyAsync(ctx->s_q + p0 * qs, qx + p0 * qs, size_t((p1 - p0) * qs),
-                        cudaMemcpyHostToDevice, cin);
-    if (e == cudaSuccess)
-      e = cudaMemcpyAsync(ctx->s_t + p0 * ts, ty + p0 * ts, size_t((p1 - p0) * ts),
-                          cudaMemcpyHostToDevice, cin);
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "H2D");
-    if (wv(cin, reinterpret_cast<unsigned long long>(ctx->progress), unsigned(w1), 0) != 0) {
+  std::vector<int64_t> wave_end;  // group-granular: group-wave boundaries
+  int64_t blk_first = 0, blk_rest = 0, nwaves = 0;
+  if (!dsp.wrap) {
+    // waves of whole stream-waves (the h-th group of every stream is group
+    // h S + st), growing 1, 1, 2, 4, 8, 8, ...
+    const int64_t waves = (G + S - 1) / S;
+    int64_t w0 = 0, step = 1;
+    while (w0 < waves) {
+      const int64_t w1 = w0 + step < waves ? w0 + step : waves;
+      wave_end.push_back(w1);
+      w0 = w1;
+      step = w0 < 2 ? 1 : (step * 2 < 8 ? step * 2 : 8);
+    }
+    nwaves = int64_t(wave_end.size());
+  } else {
+    // every stream's copy timeline (head, whole groups, tail from column
+    // ra - 32) moves in equal column blocks after a short first one, so all
+    // streams can start after ~blk_first columns of copying; the copy rate
+    // (~55 GB/s) stays ahead of the kernels' (~45 GB/s at the paper's shape)
+    blk_first = 1024;
+    blk_rest = 8192;
+    const int64_t tl = dsp.span + nt + 64;  // longest timeline
+    nwaves = 1 + (tl - blk_first + blk_rest - 1) / blk_rest;
+  }
+  auto enqueue_wave = [&](int64_t w) -> int {
+    cudaError_t ee = cudaSuccess;
+    if (!dsp.wrap) {
+      const int64_t g0w = (w == 0 ? 0 : wave_end[w - 1]) * S;
+      const int64_t p0 = g0w * 32;
+      const int64_t p1 = wave_end[w] * S * 32 < P ? wave_end[w] * S * 32 : P;
+      ee = cudaMemcpyAsync(ctx->s_q + p0 * qs, qx + p0 * qs, size_t((p1 - p0) * qs),
+                           cudaMemcpyHostToDevice, cin);
+      if (ee == cudaSuccess)
+        ee = cudaMemcpyAsync(ctx->s_t + p0 * ts, ty + p0 * ts, size_t((p1 - p0) * ts),
+                             cudaMemcpyHostToDevice, cin);
+    } else {
+      if (w == 0)
+        ee = cudaMemcpyAsync(ctx->s_q, qx, size_t(P * qs), cudaMemcpyHostToDevice, cin);
+      const int64_t x0 = w == 0 ? 0 : blk_first + (w - 1) * blk_rest;
+      const int64_t x1 = w == 0 ? blk_first : blk_first + w * blk_rest;
+      const int64_t tot = G * nt;
+      for (int64_t k = 0; k < S && ee == cudaSuccess; ++k) {
+        const int64_t V0 = k * dsp.span, V1 = V0 + dsp.span < tot ? V0 + dsp.span : tot;
+        const int64_t ga = V0 / nt, gz = V1 / nt;
+        const int64_t ra = V0 - ga * nt, rb = V1 - gz * nt;
+        const int64_t g1 = ga + (ra > 0 ? 1 : 0), nf = gz - g1;
+        // pieces: (group, first column, timeline start, columns)
+        int64_t pc[64][4];
+        int np = 0;
+        if (rb > 0) { pc[np][0] = gz; pc[np][1] = 0; pc[np][2] = 0; pc[np][3] = rb; ++np; }
+        // whole groups intersecting [x0, x1): only those, not all nf
+        {
+          const int64_t t0 = rb;
+          int64_t j0 = x0 > t0 ? (x0 - t0) / nt : 0;
+          for (int64_t j = j0; j < nf && t0 + j * nt < x1 && np < 62; ++j) {
+            pc[np][0] = g1 + j; pc[np][1] = 0; pc[np][2] = t0 + j * nt; pc[np][3] = nt; ++np;
+          }
+        }
+        if (ra > 0) {
+          pc[np][0] = ga; pc[np][1] = ra - 32; pc[np][2] = rb + nf * nt; pc[np][3] = nt - ra + 32;
+          ++np;
+        }
+        for (int i = 0; i < np && ee == cudaSuccess; ++i) {
+          const int64_t a0 = pc[i][2] > x0 ? pc[i][2] : x0;
+          const int64_t a1 = pc[i][2] + pc[i][3] < x1 ? pc[i][2] + pc[i][3] : x1;
+          if (a0 >= a1) continue;
+          const int64_t gg = pc[i][0];
+          const int64_t c_from = pc[i][1] + (a0 - pc[i][2]), c_to = c_from + (a1 - a0);
+          const int64_t rows = P - gg * 32 < 32 ? P - gg * 32 : 32;
+          // column range -> bytes of each row (2-bit packed: 4 columns per
+          // byte; the ranges are multiples of 32 columns)
+          const int64_t b0 = packed2 ? c_from / 4 : c_from;
+          const int64_t b1 = packed2 ? (c_to + 3) / 4 : c_to;
+          ee = cudaMemcpy2DAsync(ctx->s_t + gg * 32 * ts + b0, size_t(ts), ty + gg * 32 * ts + b0,
+                                 size_t(ts), size_t(b1 - b0), size_t(rows), cudaMemcpyHostToDevice,
+                                 cin);
+        }
+      }
+    }
+    if (ee != cudaSuccess) return cuda_fail(ctx, ee, "H2D");
+    if (wv(cin, reinterpret_cast<unsigned long long>(ctx->progress), unsigned(w + 1), 0) != 0) {
       cudaGetLastError();
       return BPBC_ERR_UNSUPPORTED;
     }
-    w0 = w1;
-    step = w0 < 2 ? 1 : (step * 2 < 8 ? step * 2 : 8);
-  }
-  cudaEventRecord(ctx->ev_c1, cin);
+    return BPBC_OK;
+  };
+  cudaEventRecord(ctx->ev_c0, cin);
+  if ((rc = enqueue_wave(0)) != BPBC_OK) return rc;
   RunOut o;
   o.scores = ctx->s_out;
   o.progress = ctx->progress;
+  o.blk_first = blk_first;
+  o.blk_rest = blk_rest;
   rc = run_device(ctx, dsp, ctx->s_q, ctx->s_t, P, mq, nt, c1, c2, g, o,
                   static_cast<uint8_t*>(ctx->s_ws), comp, packed2);
   if (rc != BPBC_OK) return rc;
+  for (int64_t w = 1; w < nwaves; ++w)
+    if ((rc = enqueue_wave(w)) != BPBC_OK) return rc;
+  cudaEventRecord(ctx->ev_c1, cin);
   if ((e = cudaMemcpyAsync(out_scores, ctx->s_out, size_t(P) * 4, cudaMemcpyDeviceToHost, comp)) !=
       cudaSuccess)
     return cuda_fail(ctx, e, "D2H");
@@ -905,8 +982,8 @@ int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t*
   if ((rc = make_dispatch(ctx, num_pairs, mq, nt, c1, c2, g, score_bits, kModeMax, &full)) !=
       BPBC_OK)
     return rc;
-  // fused group-granular plans: one streamed launch (host_streamed)
-  if (full.fused && !full.wrap && full.mw < 0 && !ctx->opt_chunked_host) {
+  // fused plans (group-granular or wrap-around): one streamed launch
+  if (full.fused && full.mw < 0 && !ctx->opt_chunked_host) {
     // results: straight into a pinned output, else through pinned staging
     cudaPointerAttributes pa;
     const bool pinned = cudaPointerGetAttributes(&pa, out_scores) == cudaSuccess &&

@@ -68,10 +68,14 @@ struct SweepArgs {
   int64_t span;         // columns per stream (multiple of 32, >= n)
   uint32_t* snap;       // [streams][kSnapWords][32] warp-state snapshots
   uint32_t* snap_flag;  // [streams] 1 once snapshot k is written (zeroed per call)
-  // Host-streamed inputs (fused group-granular kernel, bpbc_sw_score_batch_host):
-  // wave h (the h-th group of every stream: groups [h streams, (h+1) streams))
-  // is in device memory once *progress > h; nullptr = inputs resident.
+  // Host-streamed inputs (bpbc_sw_score_batch_host): *progress = waves the
+  // copy stream has completed; nullptr = inputs resident.  Group-granular
+  // fused kernel: wave h = the h-th group of every stream (groups
+  // [h streams, (h+1) streams)).  Wrap-around kernel: wave 0 = every query
+  // row + columns [0, blk_first) of every stream's copy timeline, wave i > 0
+  // = columns [blk_first + (i-1) blk_rest, blk_first + i blk_rest).
   const uint32_t* progress;
+  int64_t blk_first, blk_rest;
 };
 
 // Words of one lane's warp-state snapshot (wrap-around schedule): R rows x S

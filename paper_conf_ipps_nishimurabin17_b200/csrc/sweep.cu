@@ -526,13 +526,36 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
   uint32_t bad = 0;
 
   // sub-stream bookkeeping (warp-uniform): first group g0, groups touched
-  // nspan, the next target chunk (group offset yg, column ycol) and the next
-  // query group xnext with the step xth from which it may be built
-  int64_t g0 = 0, nspan = 0, yg = 0, xnext = 0, xth = 0;
+  // nspan, the next target chunk (group offset yg, column ycol, position
+  // ypos on the stream's copy timeline, whose piece ends at yend) and the
+  // next query group xnext with the step xth from which it may be built
+  int64_t g0 = 0, nspan = 0, yg = 0, xnext = 0, xth = 0, ypos = 0, yend = 0;
   int ycol = 0;
+  // host-streamed inputs (bpbc_sw_score_batch_host): the copy stream moves
+  // every stream's timeline in waves -- wave 0 = all query rows and columns
+  // [0, blk_first) of every stream, wave i = [blk_first + (i-1) blk_rest,
+  // blk_first + i blk_rest) -- and publishes the number of waves done in
+  // *progress; a chunk is read once its wave is in (warp-uniform poll)
+  uint32_t ready = a.progress ? 0u : 0xFFFFFFFFu;
+  auto wait_wave = [&](int64_t w) {
+    if (uint64_t(w) >= ready) {
+      while (true) {
+        const uint32_t v = ld_acquire_gpu(a.progress);
+        if (!__any_sync(0xFFFFFFFFu, uint64_t(v) <= uint64_t(w))) {
+          ready = v;
+          break;
+        }
+        __nanosleep(512);
+      }
+    }
+  };
   // the next 32 target columns -> ring chunk c; advance (n % 32 == 0 here)
   auto build_y = [&](int64_t c) {
     uint32_t Hw = 0, Lw = 0;
+    if (ypos < yend) {  // (chunks past the piece are never used: skip the wait)
+      const int64_t e = ypos + 32;
+      wait_wave(e <= a.blk_first ? 0 : 1 + (e - a.blk_first + a.blk_rest - 1) / a.blk_rest);
+    }
     if (yg < nspan)
       tr_load_fold(a.traw, a.tstride, a.n, (g0 + yg) * 32 + lane, a.P, ycol, packed2, Hw, Lw, bad);
     tr_butterfly(Hw, Lw, lane);
@@ -540,6 +563,7 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
     yr[slot] = make_uint2(Hw, Lw);
     yr[slot + 128] = make_uint2(Hw, Lw);
     ycol += 32;
+    ypos += 32;
     if (ycol >= a.n) {
       ycol -= a.n;
       ++yg;
@@ -547,6 +571,7 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
   };
   // query rows of group g0 + h -> x slot h & 1
   auto build_x = [&](int64_t h) {
+    wait_wave(0);  // (all query rows come with wave 0)
     int64_t g = g0 + h;
     g = g < a.G ? g : a.G - 1;
 #pragma unroll
@@ -571,6 +596,9 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
     bool snap_in = false, snap_out = false;
     int64_t steps = 0, slot = 0;
     int gs = 0;  // group ends stored
+    // (copy timeline of this stream: head [0, rb), whole groups [rb, rb +
+    // nf n), tail [rb + nf n, rb + nf n + n - ra + 32) from column ra - 32)
+    const int64_t nf = gz - (ga + (ra > 0 ? 1 : 0));
     if (sub == 0) {  // head of group gz: columns [0, rb), snapshot out
       if (rb == 0) continue;
       g0 = gz;
@@ -578,12 +606,16 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
       snap_out = true;
       slot = warp + 1;
       steps = rb;  // (a multiple of 32)
+      ypos = 0;
+      yend = rb;
     } else if (sub == 1) {  // whole groups
       g0 = ga + (ra > 0 ? 1 : 0);
       nspan = gz - g0;
       if (nspan <= 0) continue;
       gs = int(nspan);
       steps = (nspan * a.n + L + 31) / 32 * 32;
+      ypos = rb;
+      yend = rb + nf * a.n;
     } else {  // tail of group ga: columns [ra, n), snapshot in
       if (ra == 0) continue;
       g0 = ga;
@@ -593,6 +625,8 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
       snap_in = true;
       slot = warp;
       steps = (a.n - ra + L + 31) / 32 * 32;
+      ypos = rb + nf * a.n;  // chunk -1 (columns ra - 32 ..) opens the tail's range
+      yend = ypos + (a.n - ra) + 32;
     }
     // ---- fresh state (a lane enters its first group at its switch step)
     ln.reset(lane);

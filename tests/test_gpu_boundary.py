@@ -135,12 +135,21 @@ def test_host_path_chunks(pinned, packed2):
                                                             score_bits=8))
 
 
-def test_host_path_few_long_groups():
-    """Host path of a wrap-around batch (one chunk) matches the oracle."""
-    P, m, n = 600 * 32, 128, 1024
-    q, t = synth.gen_pairs(9200, P, m, n, planted=True)
-    got = bpbc.score_batch_host(q, t, 2, -1, -1, 9)
-    np.testing.assert_array_equal(got, oracle.sw_batch(q, t, 2, -1, -1, score_bits=9))
+@pytest.mark.parametrize("P,m,n,packed2", [(600 * 32, 128, 1024, False), (650 * 32 - 5, 100, 4096, True),
+                                           (32768, 128, 8192, False), (700 * 32, 200, 2048, False)])
+def test_host_path_few_long_groups(P, m, n, packed2):
+    """Host path of a wrap-around batch as one streamed launch (per-stream
+    copy timelines moved in column blocks, the wrap kernel polling the wave
+    count) matches the oracle; ragged P, padded rows, R = 8, 2-bit input."""
+    q, t = synth.gen_pairs(9200 + n, P, m, n, planted=True)
+    s = bpbc.default_score_bits(2, m, n)
+    if packed2:
+        got = bpbc.score_batch_host_packed2(synth.pack2bit(q), synth.pack2bit(t), m, n, 2, -1, -1, s)
+    else:
+        got = bpbc.score_batch_host(q, t, 2, -1, -1, s)
+    plan = bpbc.last_plan(0)
+    assert plan["wrap"] and plan["host_streamed"], plan
+    np.testing.assert_array_equal(got, oracle.sw_batch(q, t, 2, -1, -1, score_bits=s))
 
 
 def test_filter_on_side_stream():
