@@ -105,6 +105,7 @@ SweepEntry g_striped[2][kNumKinds][13];           // [mode][kind][S - 4]
 SweepEntry g_mw[2][kNumMw][kNumKinds][13];        // [mode][(R, W)][kind][S - 4]
 SweepEntry g_planes[2][kNumVariants][2][13];      // [mode][variant][rl 0..1][S - 4]
 SweepEntry g_wrap[2][kNumVariants][2][13];        // [mode][variant][rl 2..3][S - 4]
+SweepEntry g_hs[2][2][kNumRL][13];                // [mode][pad][rl][S - 4] host-streamed
 std::once_flag g_table_once;
 
 void init_table() {
@@ -113,9 +114,10 @@ void init_table() {
   memset(g_mw, 0, sizeof(g_mw));
   memset(g_planes, 0, sizeof(g_planes));
   memset(g_wrap, 0, sizeof(g_wrap));
-#define BPBC_REG(S)                                                                      \
-  register_sweep_s##S##_m0(g_table[0], g_striped[0], g_mw[0], g_planes[0], g_wrap[0]); \
-  register_sweep_s##S##_m1(g_table[1], g_striped[1], g_mw[1], g_planes[1], g_wrap[1]);
+  memset(g_hs, 0, sizeof(g_hs));
+#define BPBC_REG(S)                                                                           \
+  register_sweep_s##S##_m0(g_table[0], g_striped[0], g_mw[0], g_planes[0], g_wrap[0], g_hs[0]); \
+  register_sweep_s##S##_m1(g_table[1], g_striped[1], g_mw[1], g_planes[1], g_wrap[1], g_hs[1]);
   BPBC_REG(4)
   BPBC_REG(5)
   BPBC_REG(6)
@@ -362,7 +364,7 @@ void split_streams(const bpbc_sw_ctx* ctx, int nt, int64_t nb, int64_t nbw, Disp
 }
 
 int make_dispatch(bpbc_sw_ctx* ctx, int64_t P, int mq, int nt, int c1, int c2, int g, int S,
-                  int mode, Dispatch* d) {
+                  int mode, Dispatch* d, bool host_streamed = false) {
   int rc = make_plan(mq, c1, c2, g, S, ctx->opt_no_exact_run, ctx->opt_force_width, &d->plan);
   if (rc != BPBC_OK) return rc;
   std::call_once(g_table_once, init_table);
@@ -386,6 +388,11 @@ int make_dispatch(bpbc_sw_ctx* ctx, int64_t P, int mq, int nt, int c1, int c2, i
                        [plan.width - 4];
     }
   }
+  // host-streamed inputs: the polling instantiation of the fused kernel
+  // (the wrap kernel always polls when SweepArgs::progress is set)
+  SweepEntry hs_ent{nullptr, nullptr};
+  if (host_streamed && d->fused && plan.circuit == kExact && plan.consts == kC211)
+    hs_ent = g_hs[mode][plan.pad ? 1 : 0][plan.rl][plan.width - 4];
   if (!d->ent.launch) return BPBC_ERR_UNSUPPORTED;
   d->R = d->striped ? kStripeR : kRLR[plan.rl];
   d->L = d->striped ? 32 : kRLL[plan.rl];
@@ -408,6 +415,10 @@ int make_dispatch(bpbc_sw_ctx* ctx, int64_t P, int mq, int nt, int c1, int c2, i
     } else {
       d->mw = -1;
     }
+  }
+  if (host_streamed && d->mw < 0) {
+    if (!hs_ent.launch) return BPBC_ERR_UNSUPPORTED;  // (the caller takes the chunked path)
+    d->ent = hs_ent;
   }
   int64_t nb = occupancy_blocks(d->ent.func, threads, smem);
   if (nb < 0) return cuda_fail(ctx, cudaGetLastError(), "occupancy");
@@ -983,7 +994,10 @@ int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t*
       BPBC_OK)
     return rc;
   // fused plans (group-granular or wrap-around): one streamed launch
-  if (full.fused && full.mw < 0 && !ctx->opt_chunked_host) {
+  Dispatch hsd;
+  if (full.fused && full.mw < 0 && !ctx->opt_chunked_host &&
+      make_dispatch(ctx, num_pairs, mq, nt, c1, c2, g, score_bits, kModeMax, &hsd, true) ==
+          BPBC_OK) {
     // results: straight into a pinned output, else through pinned staging
     cudaPointerAttributes pa;
     const bool pinned = cudaPointerGetAttributes(&pa, out_scores) == cudaSuccess &&
@@ -1002,7 +1016,7 @@ int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t*
       }
       dst = ctx->h_out;
     }
-    rc = host_streamed(ctx, full, qx, ty, num_pairs, mq, nt, c1, c2, g, qs, ts, dst, packed2);
+    rc = host_streamed(ctx, hsd, qx, ty, num_pairs, mq, nt, c1, c2, g, qs, ts, dst, packed2);
     if (rc == BPBC_OK) {
       if (!pinned) memcpy(out_scores, ctx->h_out, size_t(num_pairs) * 4);
       ctx->plan_host_streamed = 1;

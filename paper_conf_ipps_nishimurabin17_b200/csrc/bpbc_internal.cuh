@@ -131,14 +131,15 @@ SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
 // short kernel, stab: [striped kind][S-4] (0 exact (+2,-1,-1), 1 saturating
 // (+2,-1,-1), 2 saturating runtime constants), ptab: [variant][rl 0..1][S-4]
 // of the planes kernel, wtab: [variant][rl - 2][S-4] of the wrap-around
-// kernel (L = 32 tilings).
+// kernel (L = 32 tilings), htab: [pad][rl][S-4] of the host-streamed fused
+// kernel (exact (+2,-1,-1) circuit; running-max objects only).
 #define BPBC_DECLARE_REG(S)                                                       \
   void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
                                 SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13], \
-                                SweepEntry (*wtab)[2][13]);                                   \
+                                SweepEntry (*wtab)[2][13], SweepEntry (*htab)[kNumRL][13]);   \
   void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
                                 SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13], \
-                                SweepEntry (*wtab)[2][13]);
+                                SweepEntry (*wtab)[2][13], SweepEntry (*htab)[kNumRL][13]);
 BPBC_DECLARE_REG(4)
 BPBC_DECLARE_REG(5)
 BPBC_DECLARE_REG(6)

@@ -6,9 +6,10 @@
 // Here a warp transposes ACROSS its lanes with the transpose of
 // transpose.cuh (shared with the fused sweep).  One warp handles one
 // (group g, 128-position chunk) item as four 32-position quarters:
-//   1. lane k loads the code bytes of pair 32g+k for all four quarters
-//      first (8 x 16-byte streaming loads, 128 B per lane in flight; 2-bit
-//      packed input: 4 x 8 B);
+//   1. the warp reads the item's 32 rows x 128 code bytes with coalesced
+//      16-byte loads (4 rows per instruction) into a shared stage, and lane
+//      k takes pair 32g+k's 128 bytes from it (ragged items: every lane
+//      loads its own row; 2-bit packed input: 4 x 8 B per lane);
 //   2. per quarter: tr_fold_u8 folds the 32 bytes into two words H, L (the
 //      high / low code bits of the 32 positions, in the fixed bit order
 //      tr_pos_u8), tr_butterfly transposes the warp's 32x32 bit matrices, so
@@ -36,10 +37,19 @@ struct PackJob {
   bool packed2;          // 4 bases per byte (bpbc_sw_score_batch_packed2)
 };
 
+// Coalesced staging of one u8 item: the 32 rows x 128 bytes of group g at
+// columns [c0, c0 + 128) are read 4 rows per instruction (8 lanes x 16 B per
+// row: 4 cache lines per load instead of 32 when every lane reads its own
+// row -- the L1 data pipe, not DRAM, limited that form) into a per-warp
+// shared buffer with 144-byte rows (conflict-free 16-byte reads below).
+constexpr int kStageRow = 32 * kPackQ + 16;
+
 __global__ void __launch_bounds__(256) pack_kernel(const PackJob j0, const PackJob j1,
                                                    int64_t num_pairs,
                                                    uint32_t* __restrict__ flags) {
+  __shared__ __align__(16) uint8_t stage[8][32 * kStageRow];  // [warp][row][byte]
   const int lane = threadIdx.x & 31;
+  uint8_t* st = stage[threadIdx.x >> 5];
   const int64_t warps = (int64_t(gridDim.x) * blockDim.x) >> 5;
   const int64_t total = j0.items + j1.items;
   uint32_t bad = 0;
@@ -71,13 +81,38 @@ __global__ void __launch_bounds__(256) pack_kernel(const PackJob j0, const PackJ
       }
       continue;
     }
-    // all four quarters are loaded before any is used (128 B per lane in flight)
     uint32_t w[kPackQ][8];
+    // whole aligned item of full rows: coalesced loads through the stage
+    const bool whole = c0 + 32 * kPackQ <= J.len && (g + 1) * 32 <= num_pairs &&
+                       (J.stride & 15) == 0 && (reinterpret_cast<uintptr_t>(J.codes) & 15) == 0;
+    if (whole) {  // warp-uniform
+      const uint8_t* src = J.codes + (g * 32) * J.stride + c0;
+      uint4 v[8];
 #pragma unroll
-    for (int h = 0; h < kPackQ; ++h) {
+      for (int i = 0; i < 8; ++i)  // rows 4i + lane / 8, bytes 16 (lane % 8)
+        v[i] = __ldcs(reinterpret_cast<const uint4*>(src + (4 * i + (lane >> 3)) * J.stride) +
+                      (lane & 7));
+      __syncwarp();  // the previous item's stage reads -> these writes
 #pragma unroll
-      for (int q = 0; q < 8; ++q) w[h][q] = 0u;
-      if (c0 + 32 * h < J.len) tr_load_u8(J.codes, J.stride, J.len, pair, num_pairs, c0 + 32 * h, w[h]);
+      for (int i = 0; i < 8; ++i)
+        *reinterpret_cast<uint4*>(st + (4 * i + (lane >> 3)) * kStageRow + 16 * (lane & 7)) = v[i];
+      __syncwarp();
+#pragma unroll
+      for (int h = 0; h < kPackQ; ++h) {  // my row (pair 32g + lane), quarter h
+        const uint4 a = *reinterpret_cast<const uint4*>(st + lane * kStageRow + 32 * h);
+        const uint4 b = *reinterpret_cast<const uint4*>(st + lane * kStageRow + 32 * h + 16);
+        w[h][0] = a.x; w[h][1] = a.y; w[h][2] = a.z; w[h][3] = a.w;
+        w[h][4] = b.x; w[h][5] = b.y; w[h][6] = b.z; w[h][7] = b.w;
+      }
+    } else {
+      // ragged / unaligned items: every lane loads its own row (all four
+      // quarters before any is used)
+#pragma unroll
+      for (int h = 0; h < kPackQ; ++h) {
+#pragma unroll
+        for (int q = 0; q < 8; ++q) w[h][q] = 0u;
+        if (c0 + 32 * h < J.len) tr_load_u8(J.codes, J.stride, J.len, pair, num_pairs, c0 + 32 * h, w[h]);
+      }
     }
     const int pos = tr_pos_u8(lane);
 #pragma unroll

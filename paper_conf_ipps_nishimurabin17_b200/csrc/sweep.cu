@@ -131,6 +131,16 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
 __device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+// Host-streamed inputs: wait until *progress > w (every lane polls; the vote
+// keeps the loop warp-uniform) and return the value seen.  Out of line: the
+// resident-input path never calls it and keeps its registers.
+__device__ __noinline__ uint32_t spin_progress(const uint32_t* progress, uint32_t w) {
+  while (true) {
+    const uint32_t v = ld_acquire_gpu(progress);
+    if (!__any_sync(0xFFFFFFFFu, v <= w)) return v;
+    __nanosleep(512);
+  }
+}
 
 // ---------------------------------------------------------------------------
 // Per-lane state and the wavefront step of the fused single-warp sweeps
@@ -333,7 +343,9 @@ struct FusedLane {
 //     2-slot shared ring at a phase start after every lane has entered the
 //     current group (and before lane 0 leaves it: needs n >= L + 32);
 //   * a __syncwarp at each phase start orders the ring writes before reads.
-template <int S, int R, int L, int CIRC, bool PAD, class K>
+// HS: host-streamed inputs (SweepArgs::progress) -- a separate instantiation,
+// so the wave polling costs the resident-input kernels no registers.
+template <int S, int R, int L, int CIRC, bool PAD, class K, bool HS = false>
 __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const K k) {
   constexpr int SEGS = 32 / L;
   constexpr int XCH = (L * R + 31) / 32;  // 32-row chunks of a group's query rows
@@ -349,28 +361,22 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   // h-th groups of all streams -- one "wave" -- are contiguous: the
   // host-streamed path copies the input wave by wave, a.progress)
   const int64_t gstr = a.streams;
+  // (every stream has base or base + 1 groups: the first rem streams one more)
   auto seg_range = [&](int s, int64_t& gbs, int64_t& gss) {
     const int64_t st = warp * SEGS + s;
     gss = 0;
     gbs = 0;
     if (st < a.streams) {
-      gss = (a.G - st + gstr - 1) / gstr;
+      gss = a.base + (st < a.rem ? 1 : 0);
       gbs = st;
     }
   };
   // host-streamed inputs: wave h (group index h of every stream) may be read
   // once the copy stream has published a.progress > h (warp-uniform poll)
-  uint32_t ready = a.progress ? 0u : 0xFFFFFFFFu;
+  uint32_t ready = 0;  // waves known to be in (HS)
   auto wait_wave = [&](int64_t h) {
-    if (uint64_t(h) >= ready) {
-      while (true) {
-        const uint32_t v = ld_acquire_gpu(a.progress);
-        if (!__any_sync(0xFFFFFFFFu, uint64_t(v) <= uint64_t(h))) {
-          ready = v;
-          break;
-        }
-        __nanosleep(512);
-      }
+    if constexpr (HS) {
+      if (uint32_t(h) >= ready) ready = spin_progress(a.progress, uint32_t(h));
     }
   };
   int64_t Gs, gb;
@@ -536,18 +542,9 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
   // [0, blk_first) of every stream, wave i = [blk_first + (i-1) blk_rest,
   // blk_first + i blk_rest) -- and publishes the number of waves done in
   // *progress; a chunk is read once its wave is in (warp-uniform poll)
-  uint32_t ready = a.progress ? 0u : 0xFFFFFFFFu;
+  uint32_t ready = a.progress ? 0u : 0xFFFFFFFFu;  // waves known to be in
   auto wait_wave = [&](int64_t w) {
-    if (uint64_t(w) >= ready) {
-      while (true) {
-        const uint32_t v = ld_acquire_gpu(a.progress);
-        if (!__any_sync(0xFFFFFFFFu, uint64_t(v) <= uint64_t(w))) {
-          ready = v;
-          break;
-        }
-        __nanosleep(512);
-      }
-    }
+    if (uint32_t(w) >= ready) ready = spin_progress(a.progress, uint32_t(w));
   };
   // the next 32 target columns -> ring chunk c; advance (n % 32 == 0 here)
   auto build_y = [&](int64_t c) {
@@ -665,6 +662,7 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
       if constexpr (BPBC_MODE == kModeThreshold) ln.flag = __ldcg(src + (R + 1) * S * 32);
       ln.cnt = int(a.n - c0) + lane;
       ln.gi = 0;
+      __syncwarp();  // build_x's ring writes (other lanes' rows) -> these reads
 #pragma unroll
       for (int r = 0; r < R; ++r) {  // (slot 0, written by build_x above)
         const uint2 v = ln.xrow[r];
@@ -1283,13 +1281,23 @@ void reg_mw(SweepEntry (*mtab)[kNumKinds][13]) {
                         (const void*)&sw_sweep_mw_kernel<S, R, W, kExact, KRun>};
 }
 
-template <int S, int R, int L, int CIRC, bool PAD, class K>
+template <int S, int R, int L, int CIRC, bool PAD, class K, bool HS = false>
 void launch_sweep(const SweepArgs& a, const KRun& kr, int grid, int block, cudaStream_t st) {
   if constexpr (K::kFixed) {
-    sw_sweep_kernel<S, R, L, CIRC, PAD, K><<<grid, block, 0, st>>>(a, K{});
+    sw_sweep_kernel<S, R, L, CIRC, PAD, K, HS><<<grid, block, 0, st>>>(a, K{});
   } else {
-    sw_sweep_kernel<S, R, L, CIRC, PAD, KRun><<<grid, block, 0, st>>>(a, kr);
+    sw_sweep_kernel<S, R, L, CIRC, PAD, KRun, HS><<<grid, block, 0, st>>>(a, kr);
   }
+}
+
+// host-streamed instantiations (exact (+2,-1,-1) circuit, running max):
+// htab[pad][rl][S - 4]
+template <int S, int RL, bool PAD>
+void reg_hs(SweepEntry (*htab)[kNumRL][13]) {
+  constexpr int R = kRLR[RL], L = kRLL[RL];
+  using K211 = KFix<2, 1, 1>;
+  htab[PAD ? 1 : 0][RL][S - 4] = {&launch_sweep<S, R, L, kExact, PAD, K211, true>,
+                                 (const void*)&sw_sweep_kernel<S, R, L, kExact, PAD, K211, true>};
 }
 
 template <int S, int CIRC, class K, int R>
@@ -1397,7 +1405,19 @@ void reg_rl(SweepEntry (*tab)[kNumRL][13]) {
 #define BPBC_REGNAME BPBC_CAT(BPBC_CAT(BPBC_CAT(register_sweep_s, BPBC_S), _m), BPBC_MODE)
 void BPBC_REGNAME(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],
                   SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13],
-                  SweepEntry (*wtab)[2][13]) {
+                  SweepEntry (*wtab)[2][13], SweepEntry (*htab)[kNumRL][13]) {
+#if BPBC_MODE == 0
+  reg_hs<BPBC_S, 0, false>(htab);
+  reg_hs<BPBC_S, 1, false>(htab);
+  reg_hs<BPBC_S, 2, false>(htab);
+  reg_hs<BPBC_S, 3, false>(htab);
+  reg_hs<BPBC_S, 0, true>(htab);
+  reg_hs<BPBC_S, 1, true>(htab);
+  reg_hs<BPBC_S, 2, true>(htab);
+  reg_hs<BPBC_S, 3, true>(htab);
+#else
+  (void)htab;
+#endif
   reg_wrap<BPBC_S, 2, false>(wtab);
   reg_wrap<BPBC_S, 2, true>(wtab);
   reg_wrap<BPBC_S, 3, false>(wtab);
