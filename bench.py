@@ -60,7 +60,7 @@ CONFIGS = {  # BASELINE.json configs; "scaling" says how N GPUs
 DEFAULT_CONFIG = 3
 CONSTS = (2, -1, -1)  # match, mismatch, gap (Table II, reading R14)
 SM_COUNT = 148
-ORACLE_FULL_SECONDS = 40.0  # full oracle parity when the estimate is below this
+ORACLE_FULL_SECONDS = 60.0  # full oracle parity when the estimate is below this
 
 
 def workload_name(cid, c):
@@ -223,6 +223,30 @@ def parity_and_cpu_baseline(q, t, got, cfg, label, sample_pairs=None):
            "sample": f"{what} of {label} (m={m}, n={n}), {dt:.1f} s on {threads} threads, "
                      f"scalar int32 DP; single thread: first {k1} pairs, {d1:.1f} s"}
     return parity, cpu
+
+
+def gathered_sample_index(P_total, m, k=65536):
+    """N > 1 parity: the seeded sample of global pair indices rank 0 checks."""
+    k = min(P_total, k)
+    rng = np.random.default_rng(P_total + m)
+    return np.sort(rng.choice(P_total, size=k, replace=False))
+
+
+def regen_pairs(seed, idx, m, n):
+    """Pairs idx (sorted global indices) of the batch: every rank generated
+    its shard with p_offset = its first global pair index, so pair p of the
+    gathered batch is gen(p_offset=p) (counter-based generator, synth/)."""
+    import synth
+    qs = np.empty((idx.size, m), dtype=np.uint8)
+    ts = np.empty((idx.size, n), dtype=np.uint8)
+    runs = np.split(idx, np.nonzero(np.diff(idx) != 1)[0] + 1) if idx.size else []
+    j = 0
+    for r in runs:
+        a, b = int(r[0]), int(r[-1]) + 1
+        qa, ta = synth.gen_pairs(seed, b - a, m, n, p_offset=a)
+        qs[j:j + b - a], ts[j:j + b - a] = qa, ta
+        j += b - a
+    return qs, ts
 
 
 def run_reference(args, cfg):
@@ -594,20 +618,9 @@ def main():
         else:
             # rank 0 regenerates a 65 536-pair sample of the WHOLE gathered
             # batch (every rank's shard) from the counter-based generator
-            k = min(P_total, 65536)
-            rng = np.random.default_rng(P_total + m)
-            idx = np.sort(rng.choice(P_total, size=k, replace=False))
-            qs = np.empty((k, m), dtype=np.uint8)
-            ts = np.empty((k, n), dtype=np.uint8)
-            # every rank generated its shard with p_offset = its first global
-            # pair index, so pair p of the gathered batch is gen(p_offset=p)
-            runs = np.split(idx, np.nonzero(np.diff(idx) != 1)[0] + 1)
-            j = 0
-            for r in runs:
-                a, b = int(r[0]), int(r[-1]) + 1
-                qa, ta = synth.gen_pairs(seed, b - a, m, n, p_offset=a)
-                qs[j:j + b - a], ts[j:j + b - a] = qa, ta
-                j += b - a
+            idx = gathered_sample_index(P_total, m)
+            qs, ts = regen_pairs(seed, idx, m, n)
+            k = idx.size
             parity, cpu = parity_and_cpu_baseline(qs, ts, got_all[idx], cfg,
                                                   f"C{args.config} (gathered over {world} ranks)",
                                                   sample_pairs=k)

@@ -73,6 +73,10 @@ typedef enum {
 
 /* Sticky device flags (bpbc_sw_get_error_flags). */
 #define BPBC_FLAG_BAD_BASE 0x1u /* a base code > 3 was packed (read as c & 3) */
+#define BPBC_FLAG_STALL 0x2u    /* a device-side wait of the host-streamed or wrap-around
+                                   schedule saw no progress for 20 s and gave up: the
+                                   scores of that call are undefined (never expected;
+                                   guards against hanging the GPU) */
 
 /* Supported ranges of this build. */
 #define BPBC_MIN_SCORE_BITS 4
@@ -264,7 +268,7 @@ int bpbc_sw_untranspose(bpbc_sw_ctx *ctx, const uint32_t *partial, int64_t num_g
 
 /* Waits for the work this ctx enqueued on every stream it used since the
  * last read (not the whole device), returns the sticky flags in *flags (bit
- * 0 = BPBC_FLAG_BAD_BASE) and clears them.  Returns BPBC_ERR_BAD_BASE when
+ * 0 = BPBC_FLAG_BAD_BASE, bit 1 = BPBC_FLAG_STALL) and clears them.  Returns BPBC_ERR_BAD_BASE when
  * that bit was set (the scores of those calls used c & 3 for the bad codes,
  * R18), BPBC_OK otherwise; *flags is written in both cases. */
 int bpbc_sw_get_error_flags(bpbc_sw_ctx *ctx, uint32_t *flags);

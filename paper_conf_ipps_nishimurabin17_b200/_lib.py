@@ -22,6 +22,7 @@ BPBC_ERR_CUDA = -3
 BPBC_ERR_OOM = -4
 BPBC_ERR_BAD_BASE = -5
 BPBC_FLAG_BAD_BASE = 0x1
+BPBC_FLAG_STALL = 0x2
 
 # name -> (restype, argtypes); must match include/bpbc_sw.h
 _c = ctypes

@@ -116,8 +116,10 @@ void init_table() {
   memset(g_wrap, 0, sizeof(g_wrap));
   memset(g_hs, 0, sizeof(g_hs));
 #define BPBC_REG(S)                                                                           \
-  register_sweep_s##S##_m0(g_table[0], g_striped[0], g_mw[0], g_planes[0], g_wrap[0], g_hs[0]); \
-  register_sweep_s##S##_m1(g_table[1], g_striped[1], g_mw[1], g_planes[1], g_wrap[1], g_hs[1]);
+  if (register_sweep_s##S##_m0)                                                              \
+    register_sweep_s##S##_m0(g_table[0], g_striped[0], g_mw[0], g_planes[0], g_wrap[0], g_hs[0]); \
+  if (register_sweep_s##S##_m1)                                                              \
+    register_sweep_s##S##_m1(g_table[1], g_striped[1], g_mw[1], g_planes[1], g_wrap[1], g_hs[1]);
   BPBC_REG(4)
   BPBC_REG(5)
   BPBC_REG(6)
@@ -929,7 +931,10 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
       }
     }
     if (ee != cudaSuccess) return cuda_fail(ctx, ee, "H2D");
-    if (wv(cin, reinterpret_cast<unsigned long long>(ctx->progress), unsigned(w + 1), 0) != 0) {
+    // the kernel's wave index: group-granular = stream-waves in (wave_end),
+    // wrap-around = column blocks in (w + 1)
+    const unsigned done = dsp.wrap ? unsigned(w + 1) : unsigned(wave_end[w]);
+    if (wv(cin, reinterpret_cast<unsigned long long>(ctx->progress), done, 0) != 0) {
       cudaGetLastError();
       return BPBC_ERR_UNSUPPORTED;
     }
@@ -954,6 +959,18 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
   if ((e = cudaStreamSynchronize(comp)) != cudaSuccess ||
       (e = cudaStreamSynchronize(cin)) != cudaSuccess)
     return cuda_fail(ctx, e, "sync");
+  // a timed-out device wait (BPBC_FLAG_STALL stays set for get_error_flags)
+  if ((e = cudaMemcpyAsync(ctx->h_flags, ctx->d_flags, sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                           comp)) != cudaSuccess ||
+      (e = cudaStreamSynchronize(comp)) != cudaSuccess)
+    return cuda_fail(ctx, e, "flags");
+  if (*ctx->h_flags & BPBC_FLAG_STALL) {  // reported here, so cleared (BAD_BASE stays)
+    *ctx->h_flags &= ~BPBC_FLAG_STALL;
+    cudaMemcpyAsync(ctx->d_flags, ctx->h_flags, sizeof(uint32_t), cudaMemcpyHostToDevice, comp);
+    cudaStreamSynchronize(comp);
+    snprintf(ctx->err, sizeof(ctx->err), "a device-side wait timed out (BPBC_FLAG_STALL)");
+    return BPBC_ERR_CUDA;
+  }
   float ms = 0;
   if (cudaEventElapsedTime(&ms, ctx->ev_c0, ctx->ev_c1) == cudaSuccess && ms > 0 &&
       P * (qs + ts) > (1 << 20))
@@ -1467,6 +1484,10 @@ int bpbc_sw_get_error_flags(bpbc_sw_ctx* ctx, uint32_t* flags) {
   if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->aux);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "get_error_flags");
   *flags = *ctx->h_flags;
+  if (*flags & BPBC_FLAG_STALL) {
+    snprintf(ctx->err, sizeof(ctx->err), "a device-side wait timed out (BPBC_FLAG_STALL)");
+    return BPBC_ERR_CUDA;
+  }
   return (*flags & BPBC_FLAG_BAD_BASE) ? BPBC_ERR_BAD_BASE : BPBC_OK;
 }
 

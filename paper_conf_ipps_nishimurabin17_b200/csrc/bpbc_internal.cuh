@@ -133,11 +133,13 @@ SweepEntry sweep_entry(int circuit, int consts, bool pad, int rl, int S);
 // of the planes kernel, wtab: [variant][rl - 2][S-4] of the wrap-around
 // kernel (L = 32 tilings), htab: [pad][rl][S-4] of the host-streamed fused
 // kernel (exact (+2,-1,-1) circuit; running-max objects only).
+// (weak: a development build may compile a subset of the widths, `make
+// WIDTHS="9 10"`; the missing widths then report BPBC_ERR_UNSUPPORTED)
 #define BPBC_DECLARE_REG(S)                                                       \
-  void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
+  __attribute__((weak)) void register_sweep_s##S##_m0(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
                                 SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13], \
                                 SweepEntry (*wtab)[2][13], SweepEntry (*htab)[kNumRL][13]);   \
-  void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
+  __attribute__((weak)) void register_sweep_s##S##_m1(SweepEntry (*tab)[kNumRL][13], SweepEntry (*stab)[13],    \
                                 SweepEntry (*mtab)[kNumKinds][13], SweepEntry (*ptab)[2][13], \
                                 SweepEntry (*wtab)[2][13], SweepEntry (*htab)[kNumRL][13]);
 BPBC_DECLARE_REG(4)

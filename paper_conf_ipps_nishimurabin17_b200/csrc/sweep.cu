@@ -131,14 +131,42 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
 __device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
-// Host-streamed inputs: wait until *progress > w (every lane polls; the vote
-// keeps the loop warp-uniform) and return the value seen.  Out of line: the
-// resident-input path never calls it and keeps its registers.
-__device__ __noinline__ uint32_t spin_progress(const uint32_t* progress, uint32_t w) {
+// Device-side waits are bounded: a wait that sees no progress for
+// kSpinTimeoutNs (a copy or a peer warp that never comes, e.g. another
+// kernel holding the SMs the wrap schedule's streams need) raises the sticky
+// BPBC_FLAG_STALL and gives up instead of hanging the GPU; the scores of
+// that call are then undefined and the host-buffer calls return
+// BPBC_ERR_CUDA.  The vote keeps every decision warp-uniform.
+constexpr uint64_t kSpinTimeoutNs = 20ull * 1000000000ull;
+__device__ __forceinline__ uint64_t global_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// Host-streamed inputs: wait until *progress > w and return the value seen
+// (0xFFFFFFFF after a timeout).  Out of line: the resident-input path never
+// calls it and keeps its registers.
+__device__ __noinline__ uint32_t spin_progress(const uint32_t* progress, uint32_t w, uint32_t* flags) {
+  const uint64_t t0 = global_ns();
   while (true) {
     const uint32_t v = ld_acquire_gpu(progress);
     if (!__any_sync(0xFFFFFFFFu, v <= w)) return v;
+    if (__any_sync(0xFFFFFFFFu, global_ns() - t0 > kSpinTimeoutNs)) {
+      if ((threadIdx.x & 31) == 0) atomicOr(flags, BPBC_FLAG_STALL);
+      return 0xFFFFFFFFu;
+    }
     __nanosleep(512);
+  }
+}
+// Wrap-around schedule: wait until the snapshot flag *f is set.
+__device__ __noinline__ void spin_flag(const uint32_t* f, uint32_t* flags) {
+  const uint64_t t0 = global_ns();
+  while (__any_sync(0xFFFFFFFFu, ld_acquire_gpu(f) == 0)) {
+    if (__any_sync(0xFFFFFFFFu, global_ns() - t0 > kSpinTimeoutNs)) {
+      if ((threadIdx.x & 31) == 0) atomicOr(flags, BPBC_FLAG_STALL);
+      return;
+    }
+    __nanosleep(256);
   }
 }
 
@@ -376,7 +404,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   uint32_t ready = 0;  // waves known to be in (HS)
   auto wait_wave = [&](int64_t h) {
     if constexpr (HS) {
-      if (uint32_t(h) >= ready) ready = spin_progress(a.progress, uint32_t(h));
+      if (uint32_t(h) >= ready) ready = spin_progress(a.progress, uint32_t(h), a.flags);
     }
   };
   int64_t Gs, gb;
@@ -544,14 +572,15 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
   // *progress; a chunk is read once its wave is in (warp-uniform poll)
   uint32_t ready = a.progress ? 0u : 0xFFFFFFFFu;  // waves known to be in
   auto wait_wave = [&](int64_t w) {
-    if (uint32_t(w) >= ready) ready = spin_progress(a.progress, uint32_t(w));
+    if (uint32_t(w) >= ready) ready = spin_progress(a.progress, uint32_t(w), a.flags);
   };
   // the next 32 target columns -> ring chunk c; advance (n % 32 == 0 here)
   auto build_y = [&](int64_t c) {
     uint32_t Hw = 0, Lw = 0;
     if (ypos < yend) {  // (chunks past the piece are never used: skip the wait)
       const int64_t e = ypos + 32;
-      wait_wave(e <= a.blk_first ? 0 : 1 + (e - a.blk_first + a.blk_rest - 1) / a.blk_rest);
+      // (wave 0 = [0, blk_first), wave i = up to blk_first + i blk_rest)
+      wait_wave(e <= a.blk_first ? 0 : (e - a.blk_first + a.blk_rest - 1) / a.blk_rest);
     }
     if (yg < nspan)
       tr_load_fold(a.traw, a.tstride, a.n, (g0 + yg) * 32 + lane, a.P, ycol, packed2, Hw, Lw, bad);
@@ -650,7 +679,7 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
     build_y(1);
     if (snap_in) {  // resume the warp state the previous stream left at column c0
       // (every lane polls; the vote keeps the loop warp-uniform)
-      while (__any_sync(0xFFFFFFFFu, ld_acquire_gpu(a.snap_flag + slot) == 0)) __nanosleep(256);
+      spin_flag(a.snap_flag + slot, a.flags);
       const uint32_t* src = a.snap + slot * (NSW * 32) + lane;
 #pragma unroll
       for (int i = 0; i < S; ++i) {

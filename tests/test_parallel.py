@@ -99,3 +99,41 @@ def test_gloo_gather_uneven_shards(tmp_path):
     path = str(tmp_path / "u.npy")
     mp.spawn(_worker_uneven, args=(2, _free_port(), path), nprocs=2, join=True)
     np.testing.assert_array_equal(np.load(path), np.arange(101, dtype=np.int32) * 7)
+
+
+def _worker_c3(rank, world, port, result_path):
+    """bench.py's strong-scaled C3 path on CPU (BASELINE configs[2]: 2^22
+    pairs sharded over the ranks): each rank generates only its
+    shard_range shard (p_offset), scores it (the oracle stands in for the
+    device here), the int32 scores are all-gathered over gloo, and rank 0
+    checks bench.py's 65 536-pair parity sample, regenerated from global pair
+    indices, against the gathered scores.  Lengths are cut to 4 x 5 so the
+    2^22 pairs stay cheap on the CPU; the pair count and the shard split are
+    C3's."""
+    import bench
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        P_total, m, n, seed = bench.CONFIGS[3]["P"], 4, 5, synth.seed_for_config(3)
+        b, e = parallel.shard_range(P_total, world, rank)
+        assert e - b == P_total // world  # 2^22 splits evenly over 2 ranks
+        q, t = synth.gen_pairs(seed, e - b, m, n, p_offset=b)
+        local = torch.from_numpy(oracle.sw_batch(q, t, 2, -1, -1, score_bits=4))
+        full = parallel.gather_scores(local, P_total).numpy()
+        if rank == 0:
+            idx = bench.gathered_sample_index(P_total, m)
+            qs, ts = bench.regen_pairs(seed, idx, m, n)
+            want = oracle.sw_batch(qs, ts, 2, -1, -1, score_bits=4)
+            np.save(result_path, np.array([idx.size, int((full[idx] != want).sum()),
+                                           full.size], dtype=np.int64))
+        dist.barrier()
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_c3_strong_shards_and_bench_parity_sample(tmp_path):
+    path = str(tmp_path / "c3.npy")
+    mp.spawn(_worker_c3, args=(2, _free_port(), path), nprocs=2, join=True)
+    k, mism, total = np.load(path)
+    assert (k, mism, total) == (65536, 0, 1 << 22)

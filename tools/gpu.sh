@@ -12,6 +12,7 @@
 #   ncupack[:ARGS]   the same for the first pack_kernel launch
 #   sanitize         compute-sanitizer memcheck/racecheck/synccheck/initcheck over tests/sanitize_run.py
 #   py:FILE[:ARGS]   python FILE ARGS
+#   sh:CMD           bash -c CMD (output in TAG_shI.log)
 set -u
 tag=$1; shift
 out=gpurun_out
@@ -25,7 +26,7 @@ for step in "$@"; do
   [ "$kind" != "$step" ] && args=${step#*:}
   echo "== [$i] $kind $args" | tee -a $out/${tag}_steps.log
   case $kind in
-    tests) timeout 2400 python -m pytest tests -m gpu -q -x --junitxml=$out/${tag}_junit.xml > $out/${tag}_tests.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
+    tests) timeout 1500 python -m pytest tests -m gpu -q --junitxml=$out/${tag}_junit.xml > $out/${tag}_tests.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
     smoke) timeout 600 python -c 'import __graft_entry__ as g; g.smoke()' > $out/${tag}_smoke.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
     bench) timeout 1800 python bench.py $args > $out/${tag}_bench$i.json 2> $out/${tag}_bench$i.err; echo "rc=$?" >> $out/${tag}_steps.log ;;
     launches) timeout 1800 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $out/${tag}_launches$i.csv python bench.py $args > $out/${tag}_launches$i.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
@@ -39,6 +40,7 @@ for step in "$@"; do
        [ "${KEEP_REP:-0}" = 1 ] || rm -f $out/${tag}_full$i.ncu-rep ;;
     sanitize) for tool in memcheck racecheck synccheck initcheck; do timeout 1200 compute-sanitizer --tool $tool python tests/sanitize_run.py > $out/${tag}_san_$tool.log 2>&1; echo "$tool rc=$?" >> $out/${tag}_steps.log; done ;;
     py) f=${args%%:*}; a=""; [ "$f" != "$args" ] && a=${args#*:}; timeout 2400 python $f $a > $out/${tag}_py$i.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
+    sh) timeout 2400 bash -c "$args" > $out/${tag}_sh$i.log 2>&1; echo "rc=$?" >> $out/${tag}_steps.log ;;
     *) echo "unknown step $kind" >> $out/${tag}_steps.log ;;
   esac
 done
