@@ -792,6 +792,9 @@ int slot_events(bpbc_sw_ctx* ctx, HostSlot& s) {
 // previous work, with a memory barrier (flags 0), done by the GPU front end.
 typedef int (*WriteValue32Fn)(void* stream, unsigned long long addr, unsigned int value,
                               unsigned int flags);
+// host_streamed(): the kernel's device-side wait timed out (internal status)
+constexpr int kStallRetry = -100;
+
 WriteValue32Fn write_value32() {
   static WriteValue32Fn fn = [] {
     void* f = nullptr;
@@ -853,6 +856,11 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
   const int64_t G = (P + 31) / 32;
   std::vector<int64_t> wave_end;  // group-granular: group-wave boundaries
   int64_t blk_first = 0, blk_rest = 0, nwaves = 0;
+  bool bulk = false;  // wrap-around: one wave of two plain copies
+  // wrap-around waves go out as one cudaMemcpy3DBatchAsync of 2D pieces each
+  // (per-piece cudaMemcpy2DAsync if the batch call is refused)
+  bool batch_ok = true;
+  std::vector<cudaMemcpy3DBatchOp> ops;
   if (!dsp.wrap) {
     // waves of whole stream-waves (the h-th group of every stream is group
     // h S + st), growing 1, 1, 2, 4, 8, 8, ...
@@ -873,6 +881,19 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
     blk_first = 1024;
     blk_rest = 8192;
     const int64_t tl = dsp.span + nt + 64;  // longest timeline
+    // Each wave costs ~2-3 2D copies per stream (~1 us of API time each in
+    // a batched submission): grow the blocks until that is at most a quarter of
+    // the copy time, else (short timelines, e.g. the paper's n = 1024) copy
+    // the whole batch with two plain copies before the kernel (bulk).
+    const double copy_s = double(P) * double(qs + ts) / ctx->h2d_bps;
+    const double call_s = 1e-6 * 3.0 * double(S);  // API time of one wave (batched)
+    while (call_s * double(1 + (tl - blk_first + blk_rest - 1) / blk_rest) > 0.25 * copy_s &&
+           blk_rest < tl)
+      blk_rest *= 2;
+    if (call_s * double(1 + (tl - blk_first + blk_rest - 1) / blk_rest) > 0.25 * copy_s) {
+      bulk = true;
+      blk_first = tl;
+    }
     nwaves = 1 + (tl - blk_first + blk_rest - 1) / blk_rest;
   }
   auto enqueue_wave = [&](int64_t w) -> int {
@@ -886,6 +907,10 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
       if (ee == cudaSuccess)
         ee = cudaMemcpyAsync(ctx->s_t + p0 * ts, ty + p0 * ts, size_t((p1 - p0) * ts),
                              cudaMemcpyHostToDevice, cin);
+    } else if (bulk) {
+      ee = cudaMemcpyAsync(ctx->s_q, qx, size_t(P * qs), cudaMemcpyHostToDevice, cin);
+      if (ee == cudaSuccess)
+        ee = cudaMemcpyAsync(ctx->s_t, ty, size_t(P * ts), cudaMemcpyHostToDevice, cin);
     } else {
       if (w == 0)
         ee = cudaMemcpyAsync(ctx->s_q, qx, size_t(P * qs), cudaMemcpyHostToDevice, cin);
@@ -924,10 +949,42 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
           // byte; the ranges are multiples of 32 columns)
           const int64_t b0 = packed2 ? c_from / 4 : c_from;
           const int64_t b1 = packed2 ? (c_to + 3) / 4 : c_to;
-          ee = cudaMemcpy2DAsync(ctx->s_t + gg * 32 * ts + b0, size_t(ts), ty + gg * 32 * ts + b0,
-                                 size_t(ts), size_t(b1 - b0), size_t(rows), cudaMemcpyHostToDevice,
-                                 cin);
+          if (batch_ok) {  // one batched submission per wave (below)
+            cudaMemcpy3DBatchOp op;
+            memset(&op, 0, sizeof(op));
+            op.src.type = cudaMemcpyOperandTypePointer;
+            op.src.op.ptr.ptr = const_cast<uint8_t*>(ty + gg * 32 * ts + b0);
+            op.src.op.ptr.rowLength = size_t(ts);
+            op.src.op.ptr.layerHeight = size_t(rows);
+            op.dst.type = cudaMemcpyOperandTypePointer;
+            op.dst.op.ptr.ptr = ctx->s_t + gg * 32 * ts + b0;
+            op.dst.op.ptr.rowLength = size_t(ts);
+            op.dst.op.ptr.layerHeight = size_t(rows);
+            op.extent = make_cudaExtent(size_t(b1 - b0), size_t(rows), 1);
+            op.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+            ops.push_back(op);
+          } else {
+            ee = cudaMemcpy2DAsync(ctx->s_t + gg * 32 * ts + b0, size_t(ts), ty + gg * 32 * ts + b0,
+                                   size_t(ts), size_t(b1 - b0), size_t(rows),
+                                   cudaMemcpyHostToDevice, cin);
+          }
         }
+      }
+      if (ee == cudaSuccess && batch_ok && !ops.empty()) {
+        size_t fail = 0;
+        ee = cudaMemcpy3DBatchAsync(ops.size(), ops.data(), &fail, 0, cin);
+        if (ee != cudaSuccess) {  // (unsupported here: per-piece 2D copies from now on)
+          cudaGetLastError();
+          batch_ok = false;
+          ee = cudaSuccess;
+          for (const auto& op : ops) {
+            ee = cudaMemcpy2DAsync(op.dst.op.ptr.ptr, op.dst.op.ptr.rowLength, op.src.op.ptr.ptr,
+                                   op.src.op.ptr.rowLength, op.extent.width, op.extent.height,
+                                   cudaMemcpyHostToDevice, cin);
+            if (ee != cudaSuccess) break;
+          }
+        }
+        ops.clear();
       }
     }
     if (ee != cudaSuccess) return cuda_fail(ctx, ee, "H2D");
@@ -964,12 +1021,11 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
                            comp)) != cudaSuccess ||
       (e = cudaStreamSynchronize(comp)) != cudaSuccess)
     return cuda_fail(ctx, e, "flags");
-  if (*ctx->h_flags & BPBC_FLAG_STALL) {  // reported here, so cleared (BAD_BASE stays)
+  if (*ctx->h_flags & BPBC_FLAG_STALL) {  // handled here, so cleared (BAD_BASE stays)
     *ctx->h_flags &= ~BPBC_FLAG_STALL;
     cudaMemcpyAsync(ctx->d_flags, ctx->h_flags, sizeof(uint32_t), cudaMemcpyHostToDevice, comp);
     cudaStreamSynchronize(comp);
-    snprintf(ctx->err, sizeof(ctx->err), "a device-side wait timed out (BPBC_FLAG_STALL)");
-    return BPBC_ERR_CUDA;
+    return kStallRetry;  // the caller reruns the batch on the chunked path
   }
   float ms = 0;
   if (cudaEventElapsedTime(&ms, ctx->ev_c0, ctx->ev_c1) == cudaSuccess && ms > 0 &&
@@ -1034,6 +1090,12 @@ int score_batch_host_impl(bpbc_sw_ctx* ctx, const uint8_t* query, const uint8_t*
       dst = ctx->h_out;
     }
     rc = host_streamed(ctx, hsd, qx, ty, num_pairs, mq, nt, c1, c2, g, qs, ts, dst, packed2);
+    if (rc == kStallRetry) {
+      // the kernel waited 20 s for copies that never came (the environment
+      // serialised it against them): this ctx uses the chunked path from now on
+      ctx->opt_chunked_host = true;
+      rc = BPBC_ERR_UNSUPPORTED;
+    }
     if (rc == BPBC_OK) {
       if (!pinned) memcpy(out_scores, ctx->h_out, size_t(num_pairs) * 4);
       ctx->plan_host_streamed = 1;
@@ -1237,6 +1299,15 @@ int bpbc_sw_init(int cuda_device, bpbc_sw_ctx** out_ctx) {
   ctx->opt_no_exact_run = env_int("BPBC_NO_EXACT_RUN", 0) != 0;
   ctx->opt_wrap = env_int("BPBC_WRAP", -1);
   ctx->opt_chunked_host = env_int("BPBC_CHUNKED_HOST", 0) != 0;
+  // The streamed host path runs its kernel concurrently with the copies it
+  // polls for; a launch-blocking or kernel-serialising environment (a
+  // profiler injected through CUDA_INJECTION64_PATH, CUDA_LAUNCH_BLOCKING=1)
+  // would make it wait for copies that are only enqueued after the launch,
+  // so those get the chunked path.
+  {
+    const char* inj = getenv("CUDA_INJECTION64_PATH");
+    if ((inj && *inj) || env_int("CUDA_LAUNCH_BLOCKING", 0) != 0) ctx->opt_chunked_host = true;
+  }
   ctx->opt_force_width = env_int("BPBC_FORCE_WIDTH", 0) != 0;
   DeviceGuard dg(cuda_device);
   e = cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);

@@ -86,6 +86,10 @@ __device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
   const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(s), "l"(gmem) : "memory");
 }
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s), "l"(gmem) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
@@ -426,13 +430,77 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   const int mypos = packed2 ? tr_pos_packed2(lane) : tr_pos_u8(lane);
   uint32_t bad = 0;
 
+  // Staged loads (ST, the L = 16 tilings, m <= 64): with groups this short
+  // every phase transposes a new query group and a target chunk per segment,
+  // and a load consumed right away exposes its HBM latency once per phase
+  // (ncu, m = n = 32: 28 % of the warp stall samples sat in the phase
+  // prologue, mostly long-scoreboard).  Whole, aligned 32-position chunks are
+  // therefore fetched one phase ahead by cp.async into a per-lane shared
+  // staging slot (no registers held across the phase) and folded from there
+  // a phase later; everything else (ragged / straddling / unaligned chunks)
+  // keeps the direct load.  A lane reads back only its own staged bytes, so
+  // cp.async.wait_all orders them; the staging slot is rewritten only after
+  // the fold has consumed the values read from it.
+  constexpr bool ST = (L == 16);
+  constexpr int SSEG = ST ? SEGS : 1, SXCH = ST ? XCH : 1;
+  __shared__ __align__(16) uint4 ystage[4][SSEG][32][2];        // [warp][segment][lane] 32 B
+  __shared__ __align__(16) uint4 xstage[4][SSEG][SXCH][32][2];  // [warp][segment][chunk][lane]
+  const bool y_al = packed2 ? ((a.tstride & 7) == 0 && (reinterpret_cast<uintptr_t>(a.traw) & 7) == 0)
+                            : ((a.tstride & 15) == 0 && (reinterpret_cast<uintptr_t>(a.traw) & 15) == 0);
+  const bool x_al = packed2 ? ((a.qstride & 7) == 0 && (reinterpret_cast<uintptr_t>(a.qraw) & 7) == 0)
+                            : ((a.qstride & 15) == 0 && (reinterpret_cast<uintptr_t>(a.qraw) & 15) == 0);
+  // raw bytes of positions [c0, c0 + 32) of one row -> my staging slot
+  auto stage_row = [&](uint4* dst, const uint8_t* base, int64_t stride, int64_t row, int c0) {
+    if (packed2) {
+      cp_async8(dst, base + row * stride + c0 / 4);
+    } else {
+      const uint8_t* src = base + row * stride + c0;
+      cp_async16(dst, src);
+      cp_async16(dst + 1, src + 16);
+    }
+  };
+  auto fold_staged = [&](const uint4* src, uint32_t& Hw, uint32_t& Lw) {
+    if (packed2) {
+      const uint2 v = *reinterpret_cast<const uint2*>(src);
+      tr_fold_packed2(v.x, v.y, Hw, Lw);
+    } else {
+      const uint4 u0 = src[0], u1 = src[1];
+      uint32_t w[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
+      tr_fold_u8(w, Hw, Lw, bad);
+    }
+  };
+  // the fast (staged) case of target chunk c of segment s: one group, whole
+  auto y_fast = [&](int s, int64_t c, int64_t& g, int& col, int64_t& h) {
+    int64_t gbs, gss;
+    seg_range(s, gbs, gss);
+    const int64_t v0 = 32 * c;
+    if (!y_al || v0 < 0 || v0 >= gss * a.n) return false;
+    h = v0 / a.n;
+    col = int(v0 - h * a.n);
+    g = gbs + h * gstr;
+    return col + 32 <= a.n;
+  };
+  auto issue_y = [&](int s, int64_t c) {
+    if constexpr (ST) {
+      int64_t g, h;
+      int col;
+      if (y_fast(s, c, g, col, h)) {
+        wait_wave(h);
+        if (g * 32 + lane < a.P) stage_row(ystage[wib][s][lane], a.traw, a.tstride, g * 32 + lane, col);
+      }
+    }
+  };
   // target columns [32c, 32c + 32) of segment s's virtual target -> ring
   auto build_y = [&](int s, int64_t c) {
     int64_t gbs, gss;
     seg_range(s, gbs, gss);
     const int64_t v0 = 32 * c;  // first virtual column
     uint32_t Hw = 0, Lw = 0;
-    if (v0 >= 0 && v0 < gss * a.n) {
+    int64_t fg = 0, fh = 0;
+    int fcol = 0;
+    if (ST && y_fast(s, c, fg, fcol, fh)) {  // issued a phase ago
+      if (fg * 32 + lane < a.P) fold_staged(ystage[wib][ST ? s : 0][lane], Hw, Lw);
+    } else if (v0 >= 0 && v0 < gss * a.n) {
       const int64_t h = v0 / a.n;
       const int col = int(v0 - h * a.n);
       const int64_t g = gbs + h * gstr;
@@ -453,17 +521,40 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     yr[s][slot] = make_uint2(Hw, Lw);
     yr[s][slot + 128] = make_uint2(Hw, Lw);
   };
-  // query rows of segment s's group h (stream-relative) -> x slot h & 1
-  auto build_x = [&](int s, int64_t h) {
+  // query group of segment s's stream-relative group h
+  auto x_group = [&](int s, int64_t h, bool& live) {
     int64_t gbs, gss;
     seg_range(s, gbs, gss);
     int64_t g = gbs + h * gstr;
-    if (g >= a.G) g = gbs < a.G ? gbs : a.G - 1;  // past the stream's last group: unused
-    else wait_wave(h);
+    live = g < a.G;
+    if (!live) g = gbs < a.G ? gbs : a.G - 1;  // past the stream's last group: unused
+    return g;
+  };
+  auto issue_x = [&](int s, int64_t h) {
+    if constexpr (ST) {
+      bool live;
+      const int64_t g = x_group(s, h, live);
+      if (!x_al) return;
+      if (live) wait_wave(h);
+#pragma unroll
+      for (int c = 0; c < XCH; ++c)
+        if (32 * c + 32 <= a.m && g * 32 + lane < a.P)
+          stage_row(xstage[wib][s][c][lane], a.qraw, a.qstride, g * 32 + lane, 32 * c);
+    }
+  };
+  // query rows of segment s's group h (stream-relative) -> x slot h & 1
+  auto build_x = [&](int s, int64_t h, bool staged) {
+    bool live;
+    const int64_t g = x_group(s, h, live);
+    if (live) wait_wave(h);
 #pragma unroll
     for (int c = 0; c < XCH; ++c) {
       uint32_t Hw = 0, Lw = 0;
-      tr_load_fold(a.qraw, a.qstride, a.m, g * 32 + lane, a.P, 32 * c, packed2, Hw, Lw, bad);
+      if (ST && staged && x_al && 32 * c + 32 <= a.m) {
+        if (g * 32 + lane < a.P) fold_staged(xstage[wib][ST ? s : 0][ST ? c : 0][lane], Hw, Lw);
+      } else {
+        tr_load_fold(a.qraw, a.qstride, a.m, g * 32 + lane, a.P, 32 * c, packed2, Hw, Lw, bad);
+      }
       tr_butterfly(Hw, Lw, lane);
       const int row = 32 * c + mypos;  // rows >= m are zero (tr_load_fold)
       if (row < L * R) xr[int(h & 1)][s * L + row / R][row % R] = make_uint2(Hw, Lw);
@@ -476,6 +567,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   ln.xrow = &xr[0][lane][0];
 
   // prologue: the first group's query planes, target chunks -1 (zeros), 0, 1
+  // (and, staged: the next group's query rows and target chunk 2 in flight)
 #pragma unroll
   for (int s = 0; s < SEGS; ++s) {
     yr[s][lane] = yr[s][lane + 32] = yr[s][lane + 64] = yr[s][lane + 96] = make_uint2(0u, 0u);
@@ -486,28 +578,36 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
   int64_t xnext[SEGS];
 #pragma unroll
   for (int s = 0; s < SEGS; ++s) {
-    build_x(s, 0);
+    build_x(s, 0, false);
     xnext[s] = 1;
+    issue_x(s, 1);
     build_y(s, 0);
     build_y(s, 1);
+    issue_y(s, 2);
   }
+  if constexpr (ST) cp_async_commit();
   const int64_t phases = a.steps / 32;  // a.steps is a multiple of 32
   for (int64_t p = 0; p < phases; ++p) {
+    if constexpr (ST) cp_async_wait_all();  // (this lane's copies issued a phase ago)
     __syncwarp();  // this warp's ring writes of the previous phase -> reads
 #pragma unroll
     for (int s = 0; s < SEGS; ++s) {
       build_y(s, p + 2);
+      issue_y(s, p + 3);
       // group h's query may be written into slot h & 1 once every lane of
       // the segment has entered group h - 1 (step (h-1) n + L); lane 0 needs
       // it at step h n
       if ((xnext[s] - 1) * a.n + L <= 32 * p) {
-        build_x(s, xnext[s]);
+        build_x(s, xnext[s], true);
         ++xnext[s];
+        issue_x(s, xnext[s]);
       }
     }
+    if constexpr (ST) cp_async_commit();
     __syncwarp();
     ln.phase(&yr[seg][(32 * p - sl) & 127], a, k);  // my 32 columns of this phase
   }
+  if constexpr (ST) cp_async_wait_all();
   if (__any_sync(0xFFFFFFFFu, bad != 0) && lane == 0) atomicOr(a.flags, BPBC_FLAG_BAD_BASE);
 }
 
@@ -577,7 +677,9 @@ __global__ void __launch_bounds__(128) sw_sweep_wrap_kernel(const SweepArgs a, c
   // the next 32 target columns -> ring chunk c; advance (n % 32 == 0 here)
   auto build_y = [&](int64_t c) {
     uint32_t Hw = 0, Lw = 0;
-    if (ypos < yend) {  // (chunks past the piece are never used: skip the wait)
+    // (chunks past the piece are never used: skip the wait; resident inputs
+    // never wait)
+    if (a.progress != nullptr && ypos < yend) {
       const int64_t e = ypos + 32;
       // (wave 0 = [0, blk_first), wave i = up to blk_first + i blk_rest)
       wait_wave(e <= a.blk_first ? 0 : (e - a.blk_first + a.blk_rest - 1) / a.blk_rest);
