@@ -856,11 +856,8 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
   const int64_t G = (P + 31) / 32;
   std::vector<int64_t> wave_end;  // group-granular: group-wave boundaries
   int64_t blk_first = 0, blk_rest = 0, nwaves = 0;
-  bool bulk = false;  // wrap-around: one wave of two plain copies
-  // wrap-around waves go out as one cudaMemcpy3DBatchAsync of 2D pieces each
-  // (per-piece cudaMemcpy2DAsync if the batch call is refused)
-  bool batch_ok = true;
-  std::vector<cudaMemcpy3DBatchOp> ops;
+  bool bulk = false;            // wrap-around, pageable inputs: two plain copies first
+  const uint8_t* ty_dev = nullptr;  // wrap-around, pinned inputs: the gather kernel's view
   if (!dsp.wrap) {
     // waves of whole stream-waves (the h-th group of every stream is group
     // h S + st), growing 1, 1, 2, 4, 8, 8, ...
@@ -877,20 +874,20 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
     // every stream's copy timeline (head, whole groups, tail from column
     // ra - 32) moves in equal column blocks after a short first one, so all
     // streams can start after ~blk_first columns of copying; the copy rate
-    // (~55 GB/s) stays ahead of the kernels' (~45 GB/s at the paper's shape)
+    // (~55 GB/s) stays ahead of the kernels' (~45 GB/s at the paper's shape).
+    // A wave is ~3 small 2D regions per stream: one launch of the gather
+    // kernel (gather.cu) reading the pinned host rows; pageable inputs (not
+    // device-readable) are copied whole before the kernel instead (bulk).
     blk_first = 1024;
     blk_rest = 8192;
     const int64_t tl = dsp.span + nt + 64;  // longest timeline
-    // Each wave costs ~2-3 2D copies per stream (~1 us of API time each in
-    // a batched submission): grow the blocks until that is at most a quarter of
-    // the copy time, else (short timelines, e.g. the paper's n = 1024) copy
-    // the whole batch with two plain copies before the kernel (bulk).
-    const double copy_s = double(P) * double(qs + ts) / ctx->h2d_bps;
-    const double call_s = 1e-6 * 3.0 * double(S);  // API time of one wave (batched)
-    while (call_s * double(1 + (tl - blk_first + blk_rest - 1) / blk_rest) > 0.25 * copy_s &&
-           blk_rest < tl)
-      blk_rest *= 2;
-    if (call_s * double(1 + (tl - blk_first + blk_rest - 1) / blk_rest) > 0.25 * copy_s) {
+    void* dp = nullptr;
+    cudaPointerAttributes pa;
+    if (cudaPointerGetAttributes(&pa, ty) == cudaSuccess && pa.type == cudaMemoryTypeHost &&
+        cudaHostGetDevicePointer(&dp, const_cast<uint8_t*>(ty), 0) == cudaSuccess && dp) {
+      ty_dev = static_cast<const uint8_t*>(dp);
+    } else {
+      cudaGetLastError();
       bulk = true;
       blk_first = tl;
     }
@@ -916,76 +913,9 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
         ee = cudaMemcpyAsync(ctx->s_q, qx, size_t(P * qs), cudaMemcpyHostToDevice, cin);
       const int64_t x0 = w == 0 ? 0 : blk_first + (w - 1) * blk_rest;
       const int64_t x1 = w == 0 ? blk_first : blk_first + w * blk_rest;
-      const int64_t tot = G * nt;
-      for (int64_t k = 0; k < S && ee == cudaSuccess; ++k) {
-        const int64_t V0 = k * dsp.span, V1 = V0 + dsp.span < tot ? V0 + dsp.span : tot;
-        const int64_t ga = V0 / nt, gz = V1 / nt;
-        const int64_t ra = V0 - ga * nt, rb = V1 - gz * nt;
-        const int64_t g1 = ga + (ra > 0 ? 1 : 0), nf = gz - g1;
-        // pieces: (group, first column, timeline start, columns)
-        int64_t pc[64][4];
-        int np = 0;
-        if (rb > 0) { pc[np][0] = gz; pc[np][1] = 0; pc[np][2] = 0; pc[np][3] = rb; ++np; }
-        // whole groups intersecting [x0, x1): only those, not all nf
-        {
-          const int64_t t0 = rb;
-          int64_t j0 = x0 > t0 ? (x0 - t0) / nt : 0;
-          for (int64_t j = j0; j < nf && t0 + j * nt < x1 && np < 62; ++j) {
-            pc[np][0] = g1 + j; pc[np][1] = 0; pc[np][2] = t0 + j * nt; pc[np][3] = nt; ++np;
-          }
-        }
-        if (ra > 0) {
-          pc[np][0] = ga; pc[np][1] = ra - 32; pc[np][2] = rb + nf * nt; pc[np][3] = nt - ra + 32;
-          ++np;
-        }
-        for (int i = 0; i < np && ee == cudaSuccess; ++i) {
-          const int64_t a0 = pc[i][2] > x0 ? pc[i][2] : x0;
-          const int64_t a1 = pc[i][2] + pc[i][3] < x1 ? pc[i][2] + pc[i][3] : x1;
-          if (a0 >= a1) continue;
-          const int64_t gg = pc[i][0];
-          const int64_t c_from = pc[i][1] + (a0 - pc[i][2]), c_to = c_from + (a1 - a0);
-          const int64_t rows = P - gg * 32 < 32 ? P - gg * 32 : 32;
-          // column range -> bytes of each row (2-bit packed: 4 columns per
-          // byte; the ranges are multiples of 32 columns)
-          const int64_t b0 = packed2 ? c_from / 4 : c_from;
-          const int64_t b1 = packed2 ? (c_to + 3) / 4 : c_to;
-          if (batch_ok) {  // one batched submission per wave (below)
-            cudaMemcpy3DBatchOp op;
-            memset(&op, 0, sizeof(op));
-            op.src.type = cudaMemcpyOperandTypePointer;
-            op.src.op.ptr.ptr = const_cast<uint8_t*>(ty + gg * 32 * ts + b0);
-            op.src.op.ptr.rowLength = size_t(ts);
-            op.src.op.ptr.layerHeight = size_t(rows);
-            op.dst.type = cudaMemcpyOperandTypePointer;
-            op.dst.op.ptr.ptr = ctx->s_t + gg * 32 * ts + b0;
-            op.dst.op.ptr.rowLength = size_t(ts);
-            op.dst.op.ptr.layerHeight = size_t(rows);
-            op.extent = make_cudaExtent(size_t(b1 - b0), size_t(rows), 1);
-            op.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-            ops.push_back(op);
-          } else {
-            ee = cudaMemcpy2DAsync(ctx->s_t + gg * 32 * ts + b0, size_t(ts), ty + gg * 32 * ts + b0,
-                                   size_t(ts), size_t(b1 - b0), size_t(rows),
-                                   cudaMemcpyHostToDevice, cin);
-          }
-        }
-      }
-      if (ee == cudaSuccess && batch_ok && !ops.empty()) {
-        size_t fail = 0;
-        ee = cudaMemcpy3DBatchAsync(ops.size(), ops.data(), &fail, 0, cin);
-        if (ee != cudaSuccess) {  // (unsupported here: per-piece 2D copies from now on)
-          cudaGetLastError();
-          batch_ok = false;
-          ee = cudaSuccess;
-          for (const auto& op : ops) {
-            ee = cudaMemcpy2DAsync(op.dst.op.ptr.ptr, op.dst.op.ptr.rowLength, op.src.op.ptr.ptr,
-                                   op.src.op.ptr.rowLength, op.extent.width, op.extent.height,
-                                   cudaMemcpyHostToDevice, cin);
-            if (ee != cudaSuccess) break;
-          }
-        }
-        ops.clear();
-      }
+      if (ee == cudaSuccess)
+        ee = launch_wrap_gather(ty_dev, ctx->s_t, P, G, nt, ts, dsp.span, S, x0, x1, packed2,
+                                ctx->num_sms, cin);
     }
     if (ee != cudaSuccess) return cuda_fail(ctx, ee, "H2D");
     // the kernel's wave index: group-granular = stream-waves in (wave_end),
