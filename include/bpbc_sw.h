@@ -45,7 +45,7 @@
  *     (give concurrent streams separate workspaces);
  *   - a ctx is not thread-safe: use one ctx per device per host thread;
  *   - the environment is read once, in bpbc_sw_init (benchmark knobs only:
- *     BPBC_MAX_BLOCKS_PER_SM, BPBC_NO_EXACT_RUN, BPBC_WRAP,
+ *     BPBC_MAX_BLOCKS_PER_SM, BPBC_MIN_BLOCKS_PER_SM, BPBC_NO_EXACT_RUN, BPBC_WRAP,
  *     BPBC_CHUNKED_HOST, BPBC_FORCE_WIDTH -- see DESIGN.md 6.4); no call on
  *     the hot path reads it.
  */

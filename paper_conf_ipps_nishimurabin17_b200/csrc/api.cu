@@ -45,6 +45,7 @@ struct bpbc_sw_ctx {
   cudaStream_t aux = nullptr;   // flag reads, frees
   // options (read once from the environment at init; benchmark knobs)
   int opt_max_blocks = 0;       // BPBC_MAX_BLOCKS_PER_SM: cap on resident sweep blocks / SM
+  int opt_min_blocks = 0;       // BPBC_MIN_BLOCKS_PER_SM: floor (with the cap: forces b)
   bool opt_no_exact_run = false;  // BPBC_NO_EXACT_RUN: exact circuit only for (+2,-1,-1)
   int opt_wrap = -1;            // BPBC_WRAP: -1 auto, 0 never, 1 whenever valid
   bool opt_chunked_host = false;  // BPBC_CHUNKED_HOST: host path always in chunks
@@ -298,7 +299,8 @@ void split_streams(const bpbc_sw_ctx* ctx, int nt, int64_t nb, int64_t nbw, Disp
   // best group-granular and best wrap-around candidates
   double gg_cost = -1.0, wr_cost = -1.0;
   int64_t gg_streams = 0, gg_steps = 0, gg_bm = 0, wr_span = 0, wr_streams = 0, wr_b = 0;
-  for (int64_t b = nb; b >= 1; --b) {
+  const int64_t bmin = ctx->opt_min_blocks > 0 && ctx->opt_min_blocks <= nb ? ctx->opt_min_blocks : 1;
+  for (int64_t b = nb; b >= bmin; --b) {
     const int64_t S = sms * b * per_block;
     {  // group-granular: stream = consecutive whole groups
       int64_t streams, gps, bm;
@@ -859,15 +861,17 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
   bool bulk = false;            // wrap-around, pageable inputs: two plain copies first
   const uint8_t* ty_dev = nullptr;  // wrap-around, pinned inputs: the gather kernel's view
   if (!dsp.wrap) {
-    // waves of whole stream-waves (the h-th group of every stream is group
-    // h S + st), growing 1, 1, 2, 4, 8, 8, ...
+    // copy waves of whole stream-waves (the h-th group of every stream is
+    // group h S + st), one stream-wave each (at most 256 copy waves): the
+    // kernel starts after the first and, when the copy is the slower side,
+    // ends one stream-wave of compute after the last byte is in (growing
+    // waves left the last, largest one's compute exposed: C2 u8 e2e 0.74 of
+    // the H2D bound)
     const int64_t waves = (G + S - 1) / S;
-    int64_t w0 = 0, step = 1;
-    while (w0 < waves) {
-      const int64_t w1 = w0 + step < waves ? w0 + step : waves;
-      wave_end.push_back(w1);
-      w0 = w1;
-      step = w0 < 2 ? 1 : (step * 2 < 8 ? step * 2 : 8);
+    const int64_t per = (waves + 255) / 256;
+    for (int64_t w1 = per; ; w1 += per) {
+      wave_end.push_back(w1 < waves ? w1 : waves);
+      if (w1 >= waves) break;
     }
     nwaves = int64_t(wave_end.size());
   } else {
@@ -1226,6 +1230,7 @@ int bpbc_sw_init(int cuda_device, bpbc_sw_ctx** out_ctx) {
   ctx->device = cuda_device;
   // benchmark knobs: read once here, never on the hot path
   ctx->opt_max_blocks = env_int("BPBC_MAX_BLOCKS_PER_SM", 0);
+  ctx->opt_min_blocks = env_int("BPBC_MIN_BLOCKS_PER_SM", 0);
   ctx->opt_no_exact_run = env_int("BPBC_NO_EXACT_RUN", 0) != 0;
   ctx->opt_wrap = env_int("BPBC_WRAP", -1);
   ctx->opt_chunked_host = env_int("BPBC_CHUNKED_HOST", 0) != 0;

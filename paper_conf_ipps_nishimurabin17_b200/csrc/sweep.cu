@@ -491,14 +491,16 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     }
   };
   // target columns [32c, 32c + 32) of segment s's virtual target -> ring
-  auto build_y = [&](int s, int64_t c) {
+  // (staged: the chunk's fast case was issued to the staging slot a phase
+  // ago; the prologue's chunks 0 and 1 are loaded directly)
+  auto build_y = [&](int s, int64_t c, bool staged) {
     int64_t gbs, gss;
     seg_range(s, gbs, gss);
     const int64_t v0 = 32 * c;  // first virtual column
     uint32_t Hw = 0, Lw = 0;
     int64_t fg = 0, fh = 0;
     int fcol = 0;
-    if (ST && y_fast(s, c, fg, fcol, fh)) {  // issued a phase ago
+    if (ST && staged && y_fast(s, c, fg, fcol, fh)) {
       if (fg * 32 + lane < a.P) fold_staged(ystage[wib][ST ? s : 0][lane], Hw, Lw);
     } else if (v0 >= 0 && v0 < gss * a.n) {
       const int64_t h = v0 / a.n;
@@ -581,8 +583,8 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     build_x(s, 0, false);
     xnext[s] = 1;
     issue_x(s, 1);
-    build_y(s, 0);
-    build_y(s, 1);
+    build_y(s, 0, false);
+    build_y(s, 1, false);
     issue_y(s, 2);
   }
   if constexpr (ST) cp_async_commit();
@@ -592,7 +594,7 @@ __global__ void __launch_bounds__(128) sw_sweep_kernel(const SweepArgs a, const 
     __syncwarp();  // this warp's ring writes of the previous phase -> reads
 #pragma unroll
     for (int s = 0; s < SEGS; ++s) {
-      build_y(s, p + 2);
+      build_y(s, p + 2, true);
       issue_y(s, p + 3);
       // group h's query may be written into slot h & 1 once every lane of
       // the segment has entered group h - 1 (step (h-1) n + L); lane 0 needs
