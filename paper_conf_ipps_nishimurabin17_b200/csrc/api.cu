@@ -72,6 +72,7 @@ struct bpbc_sw_ctx {
   void* s_ws = nullptr;
   size_t s_q_bytes = 0, s_t_bytes = 0, s_out_bytes = 0, s_ws_bytes = 0;
   uint32_t* progress = nullptr;
+  int concurrency = -1;  // streamed host path: kernels see later copy-stream writes (probe)
   cudaEvent_t ev_reset = nullptr, ev_c0 = nullptr, ev_c1 = nullptr;
   double h2d_bps = 50e9;     // measured H2D bytes/s (updated after each host call)
   double cells_ps = 5e12;    // measured cell updates/s of the device path
@@ -845,6 +846,31 @@ int host_streamed(bpbc_sw_ctx* ctx, const Dispatch& dsp, const uint8_t* qx, cons
       return cuda_fail(ctx, e, "event");
   if (!ctx->progress && (e = cudaMalloc(&ctx->progress, 256)) != cudaSuccess)
     return cuda_fail(ctx, e, "cudaMalloc(progress)");
+  // Once per ctx: can a kernel see a stream write enqueued after its launch
+  // on another stream?  (No under a kernel-serialising profiler or with
+  // launch blocking: the streamed launch would then wait for copies that
+  // are never started; BPBC_FLAG_STALL is the backstop.)
+  if (ctx->concurrency < 0) {
+    uint32_t* f = ctx->progress + 32;  // [flag, seen] in the progress block
+    if ((e = cudaMemsetAsync(f, 0, 8, comp)) != cudaSuccess ||
+        (e = cudaEventRecord(ctx->ev_reset, comp)) != cudaSuccess ||
+        (e = cudaStreamWaitEvent(cin, ctx->ev_reset, 0)) != cudaSuccess ||
+        (e = launch_probe_wait(f, f + 1, 200ull * 1000000ull, comp)) != cudaSuccess)
+      return cuda_fail(ctx, e, "concurrency probe");
+    if (wv(cin, reinterpret_cast<unsigned long long>(f), 1u, 0) != 0) {
+      cudaGetLastError();
+      return BPBC_ERR_UNSUPPORTED;
+    }
+    uint32_t seen = 0;
+    if ((e = cudaMemcpyAsync(ctx->h_flags + 1, f + 1, 4, cudaMemcpyDeviceToHost, comp)) !=
+            cudaSuccess ||
+        (e = cudaStreamSynchronize(comp)) != cudaSuccess ||
+        (e = cudaStreamSynchronize(cin)) != cudaSuccess)
+      return cuda_fail(ctx, e, "concurrency probe");
+    seen = ctx->h_flags[1];
+    ctx->concurrency = seen ? 1 : 0;
+  }
+  if (ctx->concurrency == 0) return BPBC_ERR_UNSUPPORTED;  // (the chunked path)
   // progress = 0 before the kernel starts; the copy stream's first write
   // comes after the reset (and after the allocations above)
   if ((e = cudaMemsetAsync(ctx->progress, 0, 4, comp)) != cudaSuccess ||
@@ -1234,21 +1260,13 @@ int bpbc_sw_init(int cuda_device, bpbc_sw_ctx** out_ctx) {
   ctx->opt_no_exact_run = env_int("BPBC_NO_EXACT_RUN", 0) != 0;
   ctx->opt_wrap = env_int("BPBC_WRAP", -1);
   ctx->opt_chunked_host = env_int("BPBC_CHUNKED_HOST", 0) != 0;
-  // The streamed host path runs its kernel concurrently with the copies it
-  // polls for; a launch-blocking or kernel-serialising environment (a
-  // profiler injected through CUDA_INJECTION64_PATH, CUDA_LAUNCH_BLOCKING=1)
-  // would make it wait for copies that are only enqueued after the launch,
-  // so those get the chunked path.
-  {
-    const char* inj = getenv("CUDA_INJECTION64_PATH");
-    if ((inj && *inj) || env_int("CUDA_LAUNCH_BLOCKING", 0) != 0) ctx->opt_chunked_host = true;
-  }
+
   ctx->opt_force_width = env_int("BPBC_FORCE_WIDTH", 0) != 0;
   DeviceGuard dg(cuda_device);
   e = cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
   if (e == cudaSuccess) e = cudaMalloc(&ctx->d_flags, sizeof(uint32_t));
   if (e == cudaSuccess) e = cudaMemset(ctx->d_flags, 0, sizeof(uint32_t));
-  if (e == cudaSuccess) e = cudaMallocHost(&ctx->h_flags, sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaMallocHost(&ctx->h_flags, 2 * sizeof(uint32_t));
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->buf_ev, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaDeviceSynchronize();  // the flag word is zero before any call

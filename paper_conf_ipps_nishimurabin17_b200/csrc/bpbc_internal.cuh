@@ -183,6 +183,10 @@ cudaError_t launch_wordwise(const uint8_t* q, const uint8_t* t, int64_t P, int m
 cudaError_t launch_wrap_gather(const uint8_t* host_t, uint8_t* dev_t, int64_t P, int64_t G, int n,
                                int64_t ts, int64_t span, int64_t streams, int64_t x0, int64_t x1,
                                bool packed2, int num_sms, cudaStream_t st);
+// Waits (<= timeout_ns) for *flag != 0 and writes whether it was seen
+// (gather.cu: the streamed host path's concurrency probe).
+cudaError_t launch_probe_wait(const uint32_t* flag, uint32_t* seen, uint64_t timeout_ns,
+                              cudaStream_t st);
 cudaError_t launch_extract(const uint32_t* partial, int64_t num_groups, int lanes, int s,
                            int64_t num_pairs, int32_t offset, int32_t cap, int32_t* out,
                            int num_sms, cudaStream_t stream);

@@ -104,3 +104,32 @@ cudaError_t launch_wrap_gather(const uint8_t* host_t, uint8_t* dev_t, int64_t P,
 }
 
 }  // namespace bpbc
+
+// ---------------------------------------------------------------------------
+// Concurrency probe of the streamed host path: one thread waits (at most
+// timeout_ns) for *flag to become non-zero, written by the copy stream AFTER
+// this kernel's launch, and records in *seen whether it did.  Under a
+// launch-serialising environment (a kernel profiler, CUDA_LAUNCH_BLOCKING)
+// it times out and the host path takes its chunked form instead.
+namespace bpbc {
+namespace {
+__global__ void probe_wait_kernel(const uint32_t* flag, uint32_t* seen, uint64_t timeout_ns) {
+  uint64_t t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  uint32_t v = 0;
+  do {
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
+    if (v != 0) break;
+    __nanosleep(1000);
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  } while (t - t0 < timeout_ns);
+  *seen = v != 0 ? 1u : 0u;
+}
+}  // namespace
+
+cudaError_t launch_probe_wait(const uint32_t* flag, uint32_t* seen, uint64_t timeout_ns,
+                              cudaStream_t st) {
+  probe_wait_kernel<<<1, 1, 0, st>>>(flag, seen, timeout_ns);
+  return cudaGetLastError();
+}
+}  // namespace bpbc
