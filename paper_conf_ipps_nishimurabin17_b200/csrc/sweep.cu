@@ -378,7 +378,7 @@ struct FusedLane {
 // HS: host-streamed inputs (SweepArgs::progress) -- a separate instantiation,
 // so the wave polling costs the resident-input kernels no registers.
 template <int S, int R, int L, int CIRC, bool PAD, class K, bool HS = false>
-__global__ void __launch_bounds__(128, L == 16 ? 4 : 1) sw_sweep_kernel(const SweepArgs a, const K k) {
+__global__ void __launch_bounds__(128, R <= 4 ? 4 : 3) sw_sweep_kernel(const SweepArgs a, const K k) {
   constexpr int SEGS = 32 / L;
   constexpr int XCH = (L * R + 31) / 32;  // 32-row chunks of a group's query rows
   const int lane = threadIdx.x & 31;

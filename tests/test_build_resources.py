@@ -63,7 +63,7 @@ def test_host_streamed_variants_do_not_spill(usage):
     kernels (HS = true, the host-buffer path only) may take more registers
     (the C1/C4 one: ~150, 3 blocks/SM) but never spill."""
     for pattern, _ in HEADLINE[:3]:
-        for reg, stack, shared, local in find(usage, pattern[:-3] + "1E"):
+        for reg, stack, shared, local in find(usage, pattern[:-2] + "1E"):
             assert local == 0 and stack <= 16, (pattern, reg, stack, local)
 
 
