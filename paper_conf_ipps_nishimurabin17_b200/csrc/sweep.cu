@@ -589,25 +589,147 @@ __global__ void __launch_bounds__(128, R <= 4 ? 4 : 3) sw_sweep_kernel(const Swe
   }
   if constexpr (ST) cp_async_commit();
   const int64_t phases = a.steps / 32;  // a.steps is a multiple of 32
+  if constexpr (ST) {
+    // Staged phase prologue: the target position of the next chunk to issue
+    // advances by 32 columns per phase (no 64-bit division per chunk), the
+    // chunk to build carries its fast/g decision from its issue a phase ago,
+    // and the folds of all segments' chunks come first so their butterflies
+    // form one straight-line block (the shuffle latencies overlap; ncu at
+    // m = n = 32: the per-phase transposes held 22 % of the stall samples).
+    int yi_h[SEGS], yi_col[SEGS], yb_g[SEGS];
+    bool yb_fast[SEGS];
+    const int64_t c2 = 64;  // chunk 2, issued in the prologue above
+#pragma unroll
+    for (int s = 0; s < SEGS; ++s) {
+      int64_t gbs, gss;
+      seg_range(s, gbs, gss);
+      const int h2 = int(c2 / a.n), col2 = int(c2 - int64_t(h2) * a.n);
+      yb_fast[s] = y_al && h2 < gss && col2 + 32 <= a.n;
+      yb_g[s] = int(gbs + int64_t(h2) * gstr);
+      yi_h[s] = h2;
+      yi_col[s] = col2 + 32;  // chunk 3
+      if (yi_col[s] >= a.n) {
+        yi_col[s] -= a.n;
+        ++yi_h[s];
+      }
+    }
+    constexpr int NX = SEGS * XCH;
+    for (int64_t p = 0; p < phases; ++p) {
+      cp_async_wait_all();  // (this lane's copies issued a phase ago)
+      __syncwarp();         // this warp's ring writes of the previous phase -> reads
+      // target chunk p + 2 of every segment: fold, then issue chunk p + 3
+      uint32_t yH[SEGS], yL[SEGS];
+#pragma unroll
+      for (int s = 0; s < SEGS; ++s) {
+        yH[s] = yL[s] = 0u;
+        if (yb_fast[s]) {
+          if (int64_t(yb_g[s]) * 32 + lane < a.P) fold_staged(ystage[wib][s][lane], yH[s], yL[s]);
+        } else {
+          int64_t gbs, gss;
+          seg_range(s, gbs, gss);
+          const int64_t v0 = 32 * (p + 2);
+          if (v0 < gss * a.n) {  // (ragged / straddling chunk: direct load)
+            const int64_t h = v0 / a.n;
+            const int col = int(v0 - h * a.n);
+            const int64_t g = gbs + h * gstr;
+            if (col + 32 <= a.n) {
+              wait_wave(h);
+              tr_load_fold(a.traw, a.tstride, a.n, g * 32 + lane, a.P, col, packed2, yH[s], yL[s], bad);
+            } else {
+              wait_wave(h + 1 < gss ? h + 1 : h);
+              const uint3 r3 = gather_straddle(a.traw, a.tstride, a.n, a.P, g, g + gstr,
+                                               h + 1 < gss, col, lane, packed2);
+              yH[s] = r3.x;
+              yL[s] = r3.y;
+              bad |= r3.z;
+            }
+          }
+        }
+        // issue chunk p + 3 (position advanced incrementally)
+        int64_t gbs, gss;
+        seg_range(s, gbs, gss);
+        const bool fast = y_al && yi_h[s] < gss && yi_col[s] + 32 <= a.n;
+        const int g = int(gbs + int64_t(yi_h[s]) * gstr);
+        if (fast) {
+          wait_wave(yi_h[s]);
+          if (int64_t(g) * 32 + lane < a.P)
+            stage_row(ystage[wib][s][lane], a.traw, a.tstride, int64_t(g) * 32 + lane, yi_col[s]);
+        }
+        yb_fast[s] = fast;
+        yb_g[s] = g;
+        yi_col[s] += 32;
+        if (yi_col[s] >= a.n) {
+          yi_col[s] -= a.n;
+          ++yi_h[s];
+        }
+      }
+#pragma unroll
+      for (int s = 0; s < SEGS; ++s) tr_butterfly(yH[s], yL[s], lane);
+#pragma unroll
+      for (int s = 0; s < SEGS; ++s) {
+        const int slot = int((32 * (p + 2) + mypos) & 127);
+        yr[s][slot] = make_uint2(yH[s], yL[s]);
+        yr[s][slot + 128] = make_uint2(yH[s], yL[s]);
+      }
+      // query group xnext of every segment (the segments' lanes switch at the
+      // same step offsets, so the condition is warp-uniform and equal for all
+      // segments): write slot h & 1 once every lane of the segment entered
+      // group h - 1 (step (h-1) n + L); lane 0 needs it at step h n
+      if ((xnext[0] - 1) * a.n + L <= 32 * p) {
+        uint32_t xH[NX], xL[NX];
+#pragma unroll
+        for (int s = 0; s < SEGS; ++s) {
+          bool live;
+          const int64_t g = x_group(s, xnext[s], live);
+          if (live) wait_wave(xnext[s]);
+#pragma unroll
+          for (int c = 0; c < XCH; ++c) {
+            uint32_t& H = xH[s * XCH + c];
+            uint32_t& Lw = xL[s * XCH + c];
+            H = Lw = 0u;
+            if (x_al && 32 * c + 32 <= a.m) {
+              if (g * 32 + lane < a.P) fold_staged(xstage[wib][s][c][lane], H, Lw);
+            } else {
+              tr_load_fold(a.qraw, a.qstride, a.m, g * 32 + lane, a.P, 32 * c, packed2, H, Lw, bad);
+            }
+          }
+          ++xnext[s];
+          issue_x(s, xnext[s]);
+        }
+#pragma unroll
+        for (int i = 0; i < NX; ++i) tr_butterfly(xH[i], xL[i], lane);
+#pragma unroll
+        for (int s = 0; s < SEGS; ++s) {
+#pragma unroll
+          for (int c = 0; c < XCH; ++c) {
+            const int row = 32 * c + mypos;  // rows >= m are zero
+            if (row < L * R)
+              xr[int((xnext[s] - 1) & 1)][s * L + row / R][row % R] =
+                  make_uint2(xH[s * XCH + c], xL[s * XCH + c]);
+          }
+        }
+      }
+      cp_async_commit();
+      __syncwarp();
+      ln.phase(&yr[seg][(32 * p - sl) & 127], a, k);  // my 32 columns of this phase
+    }
+  } else {
   for (int64_t p = 0; p < phases; ++p) {
-    if constexpr (ST) cp_async_wait_all();  // (this lane's copies issued a phase ago)
     __syncwarp();  // this warp's ring writes of the previous phase -> reads
 #pragma unroll
     for (int s = 0; s < SEGS; ++s) {
       build_y(s, p + 2, true);
-      issue_y(s, p + 3);
       // group h's query may be written into slot h & 1 once every lane of
       // the segment has entered group h - 1 (step (h-1) n + L); lane 0 needs
       // it at step h n
       if ((xnext[s] - 1) * a.n + L <= 32 * p) {
         build_x(s, xnext[s], true);
         ++xnext[s];
-        issue_x(s, xnext[s]);
       }
     }
-    if constexpr (ST) cp_async_commit();
     __syncwarp();
     ln.phase(&yr[seg][(32 * p - sl) & 127], a, k);  // my 32 columns of this phase
+  }
   }
   if constexpr (ST) cp_async_wait_all();
   if (__any_sync(0xFFFFFFFFu, bad != 0) && lane == 0) atomicOr(a.flags, BPBC_FLAG_BAD_BASE);
