@@ -255,3 +255,31 @@ def test_force_width_knob(s):
         os.environ.pop("BPBC_FORCE_WIDTH", None)
     assert box["plan"]["width"] == s
     np.testing.assert_array_equal(box["got"], oracle.sw_batch(q, t, 2, -1, -1, score_bits=s))
+
+
+def test_host_path_under_launch_blocking(tmp_path):
+    """With CUDA_LAUNCH_BLOCKING=1 a kernel cannot see a copy-stream write
+    enqueued after its launch: the streamed host path's once-per-ctx probe
+    (a 200 ms bounded wait) detects it and the call takes the chunked path --
+    correct scores, no stall.  Runs in a subprocess, since the
+    variable only takes effect at CUDA initialisation."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, numpy as np
+sys.path.insert(0, %r)
+import oracle, synth
+import paper_conf_ipps_nishimurabin17_b200 as bpbc
+q, t = synth.gen_pairs(9900, 20000, 128, 128, planted=True)
+got = bpbc.score_batch_host(q, t, 2, -1, -1, 9)
+plan = bpbc.last_plan(0)
+assert not plan["host_streamed"], plan
+np.testing.assert_array_equal(got, oracle.sw_batch(q, t, 2, -1, -1, score_bits=9))
+assert bpbc.get_error_flags(0) == 0
+print("OK")
+''' % os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, CUDA_LAUNCH_BLOCKING="1")
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env,
+                       timeout=600)
+    assert r.returncode == 0 and "OK" in r.stdout, r.stdout[-2000:] + r.stderr[-2000:]
