@@ -430,8 +430,9 @@ __global__ void __launch_bounds__(128, R <= 4 ? 4 : 3) sw_sweep_kernel(const Swe
   const int mypos = packed2 ? tr_pos_packed2(lane) : tr_pos_u8(lane);
   uint32_t bad = 0;
 
-  // Staged loads (ST, the L = 16 tilings, m <= 64): with groups this short
-  // every phase transposes a new query group and a target chunk per segment,
+  // Staged loads (ST: the R <= 4 tilings, m <= 128; R = 8 is register-bound):
+  // with short groups every phase transposes a new query group and a target
+  // chunk per segment,
   // and a load consumed right away exposes its HBM latency once per phase
   // (ncu, m = n = 32: 28 % of the warp stall samples sat in the phase
   // prologue, mostly long-scoreboard).  Whole, aligned 32-position chunks are
@@ -441,7 +442,7 @@ __global__ void __launch_bounds__(128, R <= 4 ? 4 : 3) sw_sweep_kernel(const Swe
   // keeps the direct load.  A lane reads back only its own staged bytes, so
   // cp.async.wait_all orders them; the staging slot is rewritten only after
   // the fold has consumed the values read from it.
-  constexpr bool ST = (L == 16);
+  constexpr bool ST = (L == 16) || (R == 4);
   constexpr int SSEG = ST ? SEGS : 1, SXCH = ST ? XCH : 1;
   __shared__ __align__(16) uint4 ystage[4][SSEG][32][2];        // [warp][segment][lane] 32 B
   __shared__ __align__(16) uint4 xstage[4][SSEG][SXCH][32][2];  // [warp][segment][chunk][lane]
