@@ -156,21 +156,25 @@ int bpbc_sw_score_batch(bpbc_sw_ctx *ctx, const uint8_t *query, const uint8_t *t
  * End-to-end variant with HOST buffers (the paper's Steps 1-5):
  * copies the inputs host->device, runs the hot path and copies the scores
  * device->host.  Plans of the fused single-warp kernel (min(m, n) <= 256)
- * run as ONE streamed launch: the inputs are copied wave by wave (a wave =
- * one 32-pair group per resident sweep stream, contiguous because the fused
- * kernel assigns groups to streams strided) on a ctx-owned copy stream, each
- * wave followed by a device-side progress write (cuStreamWriteValue32), while
- * the sweep runs concurrently on the ctx's compute stream and waits for a
- * wave's progress before reading it; only the first wave's copy is exposed.
- * Other plans (and devices without stream memory writes) cut the batch into
- * chunks of whole waves that flow through three ctx-owned buffer slots on
- * three ctx-owned streams (copy-in, kernels, copy-out), so the copy of chunk
- * c+1 and the result copy of chunk c-1 overlap the kernels of chunk c; the
- * chunk plan uses the H2D and cell rates this ctx measured on its previous
- * host call.  Batches with few groups (the wrap-around schedule) run as one
- * chunk.  Pinned inputs overlap (pageable ones are staged by the driver); a
- * pageable out_scores goes through pinned staging.  Blocking: returns when
- * out_scores is written.
+ * run as ONE streamed launch on ctx-owned streams: the sweep runs on a
+ * compute stream while the inputs are copied on a copy stream in waves, each
+ * closed by a device-side progress write (cuStreamWriteValue32) the sweep
+ * polls before it reads that wave.  Group-granular plans: a wave = one
+ * 32-pair group per sweep stream (contiguous, since groups are assigned to
+ * streams strided).  Wrap-around plans (few long groups): a
+ * wave = a column block of every stream's copy timeline, moved by one launch
+ * of a gather kernel that reads PINNED host rows directly (pageable inputs
+ * are copied whole before the sweep).  Each ctx first checks once that a
+ * kernel can see a stream write enqueued after its launch (not so under a
+ * kernel-serialising profiler or CUDA_LAUNCH_BLOCKING=1); where it cannot,
+ * and for the other plans, the batch is cut into chunks of whole waves that
+ * flow through three ctx-owned buffer slots on three ctx-owned streams
+ * (copy-in, kernels, copy-out), so the copy of chunk c+1 and the result copy
+ * of chunk c-1 overlap the kernels of chunk c; the chunk plan uses the H2D
+ * and cell rates this ctx measured on its previous host call.  Device-side
+ * waits are bounded (20 s): a wait that times out makes this ctx rerun the
+ * batch chunked.  A pageable out_scores goes through pinned staging.
+ * Blocking: returns when out_scores is written.
  *
  * query, target  host, uint8 [num_pairs][m] / [num_pairs][n].
  * out_scores     host, int32 [num_pairs].
